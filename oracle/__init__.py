@@ -1,0 +1,231 @@
+"""ConVGPU scheduler-replay ORACLE — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+`--impl reference` leg may import this package.  It wraps the plain C oracle
+(oracle/oracle.c, built into oracle/liboracle.so with gcc) through ctypes and
+ships an independent pure-Python brute-force explorer (oracle/bruteforce.py).
+It never imports the product package and the product never imports it.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = [os.path.join(_HERE, "oracle.c")]
+
+POLICY = {"fifo": 0, "best_fit": 1, "recent_fit": 2, "random_fit": 3}
+NONE32 = 0xFFFFFFFF
+NONE8 = 0xFF
+FLAG_BITS = ("deadlock", "overcommit", "invalid_limit", "invalid_free",
+             "unsorted_arrival", "tick_range", "bad_program")
+
+
+def build(force: bool = False) -> str:
+    """Compile the C oracle with gcc (plain -O2, no special tuning)."""
+    newest = max(os.path.getmtime(p) for p in _SRC + [os.path.join(_HERE, "oracle.h")])
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < newest:
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-fPIC", "-shared",
+                               "-o", _SO] + _SRC)
+        exe = os.path.join(_HERE, "oracle_run")
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-o", exe,
+                               os.path.join(_HERE, "oracle_run.c"), _SRC[0]])
+    return _SO
+
+
+class _Trace(C.Structure):
+    _fields_ = [("n", C.c_uint32), ("K", C.c_uint32),
+                ("arrival", C.POINTER(C.c_uint32)), ("limit", C.POINTER(C.c_uint32)),
+                ("delta", C.POINTER(C.c_uint32)), ("arg", C.POINTER(C.c_uint32))]
+
+
+class _Result(C.Structure):
+    _fields_ = [("admit_tick", C.c_uint32 * 64), ("admit_rank", C.c_uint32 * 64),
+                ("wait", C.c_uint32 * 64), ("finish", C.c_uint32 * 64),
+                ("makespan", C.c_uint32), ("peak_reserved", C.c_uint32),
+                ("peak_used", C.c_uint32), ("flags", C.c_uint32),
+                ("sum_wait", C.c_uint64), ("n_rejected", C.c_uint32),
+                ("n_select", C.c_uint32), ("digest", C.c_uint64),
+                ("events", C.c_uint64), ("violation", C.c_int32),
+                ("violation_event", C.c_uint64)]
+
+
+class Stats(C.Structure):
+    _fields_ = [("traces", C.c_uint64), ("events", C.c_uint64),
+                ("sum_makespan", C.c_uint64), ("sum_wait", C.c_uint64),
+                ("n_rejected", C.c_uint64), ("n_select", C.c_uint64),
+                ("digest_sum", C.c_uint64), ("max_makespan", C.c_uint32),
+                ("max_peak_reserved", C.c_uint32), ("flag_count", C.c_uint32 * 8)]
+
+    def as_dict(self) -> dict:
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "flag_count"}
+        d["flag_count"] = list(self.flag_count)
+        return d
+
+
+class _Gen(C.Structure):
+    _fields_ = [("gen_seed", C.c_uint64), ("n", C.c_uint32), ("K", C.c_uint32),
+                ("n_classes", C.c_uint32), ("class_mib", C.c_uint32 * 8),
+                ("num", C.c_uint32), ("den", C.c_uint32), ("iat", C.c_uint32),
+                ("dur_base", C.c_uint32), ("dur_step", C.c_uint32),
+                ("dur_class_offset", C.c_uint32), ("dur_jit", C.c_uint32),
+                ("ovh", C.c_uint32)]
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = C.CDLL(_SO)
+        u32p, u64p, u8p = C.POINTER(C.c_uint32), C.POINTER(C.c_uint64), C.POINTER(C.c_uint8)
+        L.orc_philox4x32_10.argtypes = [u32p, u32p, u32p]
+        L.orc_mix64.argtypes = [C.c_uint64]
+        L.orc_mix64.restype = C.c_uint64
+        L.orc_replay.argtypes = [C.POINTER(_Trace), C.c_uint32, C.c_int, C.c_uint64,
+                                 C.c_uint64, C.c_uint32, C.c_int, C.POINTER(_Result)]
+        L.orc_generate.argtypes = [C.POINTER(_Gen), C.c_uint64, u32p, u32p, u32p, u32p]
+        L.orc_replay_range.argtypes = [C.POINTER(_Gen), C.c_uint32, C.c_int, C.c_uint64,
+                                       C.c_uint32, C.c_uint64, C.c_uint64, C.c_int,
+                                       C.POINTER(Stats), u32p, u64p, u32p, u32p, u8p,
+                                       u32p, u32p]
+        L.orc_replay_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, u32p, u32p,
+                                       u32p, u32p, C.c_uint32, C.c_int, C.c_uint64,
+                                       C.c_uint64, C.c_uint32, C.c_int, C.POINTER(Stats),
+                                       u32p, u64p, u32p, u32p, u8p, u32p, u32p]
+        _lib = L
+    return _lib
+
+
+def _p(a, ct=C.c_uint32):
+    return None if a is None else a.ctypes.data_as(C.POINTER(ct))
+
+
+def _pol(policy) -> int:
+    return POLICY[policy] if isinstance(policy, str) else int(policy)
+
+
+def philox4x32_10(ctr, key):
+    c = np.ascontiguousarray(ctr, np.uint32)
+    k = np.ascontiguousarray(key, np.uint32)
+    out = np.zeros(4, np.uint32)
+    lib().orc_philox4x32_10(_p(c), _p(k), _p(out))
+    return [int(x) for x in out]
+
+
+def mix64(z: int) -> int:
+    return int(lib().orc_mix64(z & 0xFFFFFFFFFFFFFFFF))
+
+
+def replay_trace(arrival, limit, delta, arg, cap, policy, tid=0, seed=0, ovh=0,
+                 check=True) -> dict:
+    """Replay one trace.  delta/arg are [K][n]."""
+    arrival = np.ascontiguousarray(arrival, np.uint32)
+    limit = np.ascontiguousarray(limit, np.uint32)
+    delta = np.ascontiguousarray(delta, np.uint32)
+    arg = np.ascontiguousarray(arg, np.uint32)
+    n = arrival.shape[0]
+    K = delta.shape[0]
+    tr = _Trace(n, K, _p(arrival), _p(limit), _p(delta), _p(arg))
+    res = _Result()
+    rc = lib().orc_replay(C.byref(tr), cap, _pol(policy), tid, seed, ovh,
+                          1 if check else 0, C.byref(res))
+    if rc:
+        raise ValueError(f"orc_replay rc={rc}")
+    out = {f: getattr(res, f) for f, _ in _Result._fields_}
+    for f in ("admit_tick", "admit_rank", "wait", "finish"):
+        out[f] = list(out[f])[:n]
+    return out
+
+
+def gen_struct(g) -> _Gen:
+    cm = (C.c_uint32 * 8)(*list(g.class_mib) + [0] * (8 - len(g.class_mib)))
+    return _Gen(g.gen_seed, g.n, g.K, len(g.class_mib), cm, g.num, g.den, g.iat,
+                g.dur_base, g.dur_step, g.dur_class_offset, g.dur_jit, g.ovh)
+
+
+def generate(g, tid: int):
+    n, K = g.n, g.K
+    arrival = np.zeros(n, np.uint32); limit = np.zeros(n, np.uint32)
+    delta = np.zeros((K, n), np.uint32); arg = np.zeros((K, n), np.uint32)
+    rc = lib().orc_generate(C.byref(gen_struct(g)), tid, _p(arrival), _p(limit),
+                            _p(delta), _p(arg))
+    if rc:
+        raise ValueError("orc_generate rc=%d" % rc)
+    return arrival, limit, delta, arg
+
+
+def generate_batch(g, tid_lo: int, count: int):
+    """Oracle-side generation of a batch in the C-ABI layout ([N,n], [N,K,n])."""
+    n, K = g.n, g.K
+    A = np.zeros((count, n), np.uint32); Lm = np.zeros((count, n), np.uint32)
+    D = np.zeros((count, K, n), np.uint32); R = np.zeros((count, K, n), np.uint32)
+    gs = gen_struct(g)
+    for i in range(count):
+        rc = lib().orc_generate(C.byref(gs), tid_lo + i, _p(A[i]), _p(Lm[i]), _p(D[i]), _p(R[i]))
+        if rc:
+            raise ValueError("orc_generate rc=%d" % rc)
+    return A, Lm, D, R
+
+
+def _outputs(count, n, full):
+    o = dict(sum_u32x4=np.zeros((count, 4), np.uint32), sum_u64x2=np.zeros((count, 2), np.uint64),
+             cnt_u32x2=np.zeros((count, 2), np.uint32))
+    if full:
+        o.update(admit_tick=np.zeros((count, n), np.uint32),
+                 admit_rank=np.zeros((count, n), np.uint8),
+                 wait=np.zeros((count, n), np.uint32), finish=np.zeros((count, n), np.uint32))
+    else:
+        o.update(admit_tick=None, admit_rank=None, wait=None, finish=None)
+    return o
+
+
+def _pack(o, st):
+    s = o["sum_u32x4"]; w = o["sum_u64x2"]; cnt = o["cnt_u32x2"]
+    res = dict(stats=st.as_dict(), makespan=s[:, 0], peak_reserved=s[:, 1],
+               peak_used=s[:, 2], flags=s[:, 3], sum_wait=w[:, 0], digest=w[:, 1],
+               n_rejected=cnt[:, 0], n_select=cnt[:, 1])
+    for f in ("admit_tick", "admit_rank", "wait", "finish"):
+        if o[f] is not None:
+            res[f] = o[f]
+    return res
+
+
+def replay_range(w, policy, tid_lo: int, tid_hi: int, full: bool = False,
+                 check: bool = False, rand_seed=None):
+    """Generate + replay global trace ids [tid_lo, tid_hi) of workload w."""
+    g = w.gen
+    count = tid_hi - tid_lo
+    o = _outputs(count, g.n, full)
+    st = Stats()
+    seed = w.rand_seed if rand_seed is None else rand_seed
+    rc = lib().orc_replay_range(C.byref(gen_struct(g)), w.cap, _pol(policy), seed, w.ovh,
+                                tid_lo, tid_hi, 1 if check else 0, C.byref(st),
+                                _p(o["sum_u32x4"]), _p(o["sum_u64x2"], C.c_uint64),
+                                _p(o["cnt_u32x2"]), _p(o["admit_tick"]),
+                                _p(o["admit_rank"], C.c_uint8), _p(o["wait"]), _p(o["finish"]))
+    res = _pack(o, st)
+    res["rc"] = rc
+    return res
+
+
+def replay_batch(b, cap, policy, tid_base=0, rand_seed=0, ovh=0, check=False, full=True):
+    """Replay a workloads.Batch (numpy) with the oracle."""
+    count, n, K = b.count, b.n, b.K
+    o = _outputs(count, n, full)
+    st = Stats()
+    arrs = [np.ascontiguousarray(x, np.uint32) for x in (b.arrival, b.limit, b.delta, b.arg)]
+    rc = lib().orc_replay_batch(n, K, count, *[_p(x) for x in arrs], cap, _pol(policy),
+                                tid_base, rand_seed, ovh, 1 if check else 0, C.byref(st),
+                                _p(o["sum_u32x4"]), _p(o["sum_u64x2"], C.c_uint64),
+                                _p(o["cnt_u32x2"]), _p(o["admit_tick"]),
+                                _p(o["admit_rank"], C.c_uint8), _p(o["wait"]), _p(o["finish"]))
+    res = _pack(o, st)
+    res["rc"] = rc
+    return res
