@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""bench.py — events replayed per second by the B200 replay of ConVGPU's
+GPU-memory scheduler (BASELINE.json metric), one JSON line on rank 0.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Workload (N=1): BASELINE.json configs[2] — 10^6 traces x 64 containers, 2x
+oversubscription of a 180 GiB GPU (workloads.CONFIGS["c2"]).  Under torchrun
+(N>1) every rank replays its own 10^6-trace shard of the global id space
+(weak scaling; config [3]'s sharding) and the per-policy statistics are
+all-reduced over NCCL each step.  A "step" = the whole hot path over the
+batch: replay under FIFO, Best-Fit, Recent-Fit and Random-Fit (4 launches of
+the replay kernel, full per-container outputs + summaries + statistics).
+Inputs (2.56 GB per rank) are resident in HBM before the timed region and are
+larger than the 126 MB L2, so no flush is needed between steps.
+
+`--impl reference` times the C oracle (test infrastructure, the only
+reference this paper-only task has) on the host cores on a bounded sample of
+the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "scheduler events replayed/sec per policy at 1/2/4/8 B200 (% HBM roofline)"
+POLICIES = W.POLICIES
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c2", choices=["c1", "c2", "mimic"])
+    ap.add_argument("--traces", type=int, default=None, help="traces per GPU (default: config)")
+    ap.add_argument("--outputs", default="full", choices=["full", "summary"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=32768, help="traces per policy (cpu leg)")
+    ap.add_argument("--ref-sample", type=int, default=4096, help="traces per policy per step (reference arm)")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu: no sampler/e2e/cpu")
+    return ap.parse_args()
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0)),
+            int(os.environ.get("WORLD_SIZE", 1)))
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.rows = []
+        self.proc = None
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except FileNotFoundError:
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+        time.sleep(0.3)
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.thread.join(timeout=2)
+        sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            if len(r) < 9:
+                continue
+            for name, v in zip(names, r[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        loaded = [s for s in sm if s > 0.5 * (max(mx) if mx else 1)] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(self.rows), "samples_under_load": len(loaded)}
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    """The oracle (plain single-threaded C) timed on this host's cores."""
+    if rank != 0:
+        return
+    import oracle
+    w = W.CONFIGS[args.workload]
+    S = args.ref_sample
+    oracle.build()
+    oracle.lib()
+    times = []
+    events = 0
+    for step in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        ev = 0
+        for p in POLICIES:
+            r = oracle.replay_range(w, p, 0, S)
+            ev += r["stats"]["events"]
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+            events += ev
+    total = sum(times)
+    value = events / total
+    sample = f"{S} traces x {len(POLICIES)} policies per step of {w.name} (ids 0..{S - 1})"
+    out = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "events/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * total / len(times), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": w.name, "traces_per_step": S, "containers": w.gen.n,
+                   "ops_per_container": w.gen.K, "capacity_mib": w.cap,
+                   "policies": list(POLICIES)},
+        "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+
+
+# ------------------------------------------------------------------ our arm
+def cpu_baseline(w, sample):
+    import oracle
+    oracle.build()
+    t0 = time.perf_counter()
+    ev = 0
+    for p in POLICIES:
+        ev += oracle.replay_range(w, p, 0, sample)["stats"]["events"]
+    dt = time.perf_counter() - t0
+    return {"value": ev / dt, "unit": "events/s", "cores": 1, "kind": "oracle",
+            "sample": f"{sample} traces x {len(POLICIES)} policies of {w.name} "
+                      f"(ids 0..{sample - 1}), single-threaded C oracle, {dt:.1f} s"}
+
+
+def traffic_from_profiles(workload, traces):
+    """dram bytes per replay launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_full_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        if d.get("workload") == workload and int(d.get("traces")) == traces:
+            return d.get("dram_bytes_per_launch")
+    except Exception:
+        pass
+    return None
+
+
+def run_ours(args, rank, local_rank, world):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_kangjkkk17_b200 as cg
+    from paper_conf_cluster_kangjkkk17_b200 import dist as cgd
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cg.lib()
+    w = W.CONFIGS[args.workload]
+    Nr = args.traces or (w.n_traces if args.workload != "c3" else w.n_traces // world)
+    n, K = w.gen.n, w.gen.K
+    base = rank * Nr  # rank r owns global ids [r*Nr, (r+1)*Nr)
+    stream = torch.cuda.current_stream()
+
+    # a0: generation (timed separately, not part of events/s)
+    g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    g0.record()
+    tr = cg.generate(w.gen, base, Nr, device=dev)
+    g1.record()
+    torch.cuda.synchronize()
+    gen_ms = g0.elapsed_time(g1)
+
+    full = args.outputs == "full"
+    outs = {p: cg.alloc_out(Nr, n, device=dev, full=full, stats=False) for p in POLICIES}
+    nsteps = args.warmup + args.steps
+    stats = {p: torch.zeros(nsteps, 12, dtype=torch.int64, device=dev) for p in POLICIES}
+    ev_s = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
+    ev_e = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
+
+    def step(s, timed_idx=None):
+        for p in POLICIES:
+            o = outs[p]
+            o.stats = stats[p][s]
+            if timed_idx is not None:
+                ev_s[p][timed_idx].record(stream)
+            cg.replay(tr, w.cap, p, o, rand_seed=w.rand_seed, ovh=w.ovh, stream=stream)
+            if timed_idx is not None:
+                ev_e[p][timed_idx].record(stream)
+            if world > 1:
+                cgd.reduce_stats(stats[p][s])
+
+    for s in range(args.warmup):
+        step(s)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    sampler = None
+    if not args.profile:
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        phys = int(vis.split(",")[local_rank]) if vis else local_rank
+        sampler = ClockSampler(phys)
+        sampler.start()
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t_start.record(stream)
+    for k in range(args.steps):
+        step(args.warmup + k, k)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop() if sampler else None
+    ms_local = t_start.elapsed_time(t_end)
+    ms = cgd.max_over_ranks(ms_local, dev)
+
+    per_trace_events = n * (1 + K)
+    # correctness of the timed work: every timed launch replayed every trace
+    last = args.warmup + args.steps - 1
+    checks = {}
+    for p in POLICIES:
+        st = cg.stats_dict(stats[p][last].cpu().numpy().view(cg.STATS_DTYPE)[0])
+        exp_ev = Nr * per_trace_events * (world if world > 1 else 1)
+        assert st["events"] == exp_ev, (p, st["events"], exp_ev)
+        assert st["flag_count"] == [0] * 8, (p, st["flag_count"])
+        checks[p] = st
+    launch_ms = {p: statistics.mean(ev_s[p][k].elapsed_time(ev_e[p][k]) for k in range(args.steps))
+                 for p in POLICIES}
+
+    events_total = world * args.steps * len(POLICIES) * Nr * per_trace_events
+    value = events_total / (ms / 1e3)
+
+    # roofline of the replay kernel (dominant kernel)
+    in_b = n * (2 + 2 * K) * 4
+    out_b = (n * 13 if full else 0) + 40
+    bytes_per_launch = Nr * (in_b + out_b)
+    avg_launch_s = statistics.mean(launch_ms.values()) / 1e3
+    peak, peak_src = measured_peak()
+    achieved = bytes_per_launch / avg_launch_s / 1e9
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": traffic_from_profiles(w.name, Nr),
+                "kernel": "convgpu::replay_kernel", "algorithmic_bytes_per_launch": bytes_per_launch,
+                "bytes_per_event": (in_b + out_b) / per_trace_events, "peak_source": peak_src,
+                "avg_launch_ms": avg_launch_s * 1e3,
+                "note": "issue/latency-bound warp-serial event loop; see DESIGN.md §Roofline"}
+
+    result = None
+    if rank == 0:
+        result = {
+            "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": w.name + " (BASELINE configs[%s])" % {"c1": 1, "c2": 2}.get(args.workload, "-"),
+                       "traces_per_gpu": Nr, "containers": n, "ops_per_container": K,
+                       "capacity_mib": w.cap, "policies": list(POLICIES), "outputs": args.outputs,
+                       "global_trace_ids": f"[r*{Nr}, (r+1)*{Nr}) per rank r",
+                       "l2": "inputs %.2f GB per rank > 126 MB L2; no flush" % (Nr * in_b / 1e9),
+                       "parallelism": f"dp{world} (trace-id shards, NCCL stats all-reduce)"},
+            "per_policy": {p: {"events_per_s": Nr * per_trace_events * world / (launch_ms[p] / 1e3),
+                               "launch_ms": launch_ms[p],
+                               "digest_sum": "%016x" % (checks[p]["digest_sum"] & (2**64 - 1)),
+                               "sum_wait": checks[p]["sum_wait"],
+                               "sum_makespan": checks[p]["sum_makespan"]} for p in POLICIES},
+            "gen_ms": gen_ms,
+            "roofline": roofline,
+            "gpu_launches": args.steps * len(POLICIES) * cg.lib().convgpu_launches_per_call(),
+            "clocks": clocks,
+        }
+
+    # e2e: the same metric through the host-memory C-ABI entry point
+    if not args.no_e2e and not args.profile:
+        chunk = 1 << 17
+        hbuf = [torch.empty(t.shape, dtype=torch.int32, pin_memory=True)
+                for t in (tr.arrival, tr.limit, tr.op_delta, tr.op_arg)]
+        for h, t in zip(hbuf, (tr.arrival, tr.limit, tr.op_delta, tr.op_arg)):
+            h.copy_(t)
+        del outs
+        torch.cuda.empty_cache()
+        import numpy as np
+        hsum_t = torch.empty(len(POLICIES) * Nr * 5, dtype=torch.int64, pin_memory=True)
+        hsum = hsum_t.numpy().view(cg.SUMMARY_DTYPE).reshape(len(POLICIES), Nr)
+        ws = torch.empty(cg.host_workspace_bytes(n, K, chunk, len(POLICIES)), dtype=torch.uint8,
+                         device=dev)
+        cg.replay_host(*hbuf, w.cap, POLICIES, trace_id_base=base, rand_seed=w.rand_seed,
+                       ovh=w.ovh, chunk=chunk, summary=hsum, workspace=ws, stream=stream)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            st_host = cg.replay_host(*hbuf, w.cap, POLICIES, trace_id_base=base,
+                                     rand_seed=w.rand_seed, ovh=w.ovh, chunk=chunk,
+                                     summary=hsum, workspace=ws, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = cgd.max_over_ranks(e0.elapsed_time(e1), dev)
+        for q, p in enumerate(POLICIES):
+            assert int(st_host[q]["events"]) == Nr * per_trace_events
+            if rank == 0 and world == 1:
+                assert "%016x" % int(st_host[q]["digest_sum"]) == result["per_policy"][p]["digest_sum"]
+        if rank == 0:
+            result["e2e"] = {
+                "value": world * args.e2e_steps * len(POLICIES) * Nr * per_trace_events / (e2e_ms / 1e3),
+                "unit": "events/s", "steps": args.e2e_steps,
+                "h2d_bytes_per_step": Nr * in_b,
+                "d2h_bytes_per_step": len(POLICIES) * (Nr * 40 + 96),
+                "api": "convgpu_replay_host (pinned host buffers, %d-trace chunks, copy/compute overlap)" % chunk,
+            }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
+        result["cpu_baseline"] = cpu_baseline(w, args.cpu_sample)
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    rank, local_rank, world = env_rank()
+    if world != args.gpus and not (world == 1 and args.gpus == 1):
+        if world == 1:
+            sys.stderr.write("bench.py: --gpus %d needs torchrun with %d ranks\n" % (args.gpus, args.gpus))
+            sys.exit(2)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    run_ours(args, rank, local_rank, world)
+
+
+if __name__ == "__main__":
+    main()

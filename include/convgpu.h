@@ -1,0 +1,217 @@
+/*
+ * convgpu.h — C ABI of the B200-native batched replay of ConVGPU's
+ * GPU-memory scheduler (Kang, Jun, Kim, Kim, Kim, "ConVGPU: GPU Management
+ * Middleware in Container Based Virtualized Environment", IEEE CLUSTER 2017;
+ * text in PAPER.md, cited "P:<line>").  DESIGN.md states the semantics and
+ * every reading ("R<n>") of the paper that the kernels implement.
+ *
+ * Library: paper_conf_cluster_kangjkkk17_b200/libconvgpu.so (sm_100a only).
+ *
+ * Conventions for every entry point
+ *  - Pointers named "device" must be caller-owned device (or managed)
+ *    memory on the current CUDA device; the library never allocates, frees
+ *    or retains them.  Host-side structs are read during the call only.
+ *  - Work is enqueued on the caller's stream (`stream`, a cudaStream_t; NULL =
+ *    the legacy default stream) and is asynchronous: results are valid after
+ *    the caller synchronises that stream.
+ *  - Return 0 on success or a negative errno-style code:
+ *      -EINVAL (-22) invalid argument (NULL required pointer, host pointer
+ *                    where device memory is required, size out of range),
+ *      -ENODEV (-19) the current device is not an sm_100 B200-class GPU,
+ *      -EIO    (-5)  a CUDA error; its text is kept per thread and returned
+ *                    by convgpu_strerror(-EIO).
+ *  - No global mutable state: calls are reentrant and thread-safe; calls on
+ *    different streams / devices may run concurrently.
+ *  - Data-level anomalies are never return codes: they are per-trace flag
+ *    bits (CONVGPU_FLAG_*) in the outputs.
+ */
+#ifndef CONVGPU_H
+#define CONVGPU_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CONVGPU_ABI_VERSION 1
+#define CONVGPU_MAX_CONTAINERS 64u   /* containers per trace */
+#define CONVGPU_MAX_OPS 8u           /* ops per container (K) */
+#define CONVGPU_CAPACITY_LIMIT (1u << 26) /* capacity_mib must be below this */
+#define CONVGPU_OVERHEAD_LIMIT (1u << 30) /* ctx_overhead_mib must be below this */
+#define CONVGPU_TICK_LIMIT (1u << 26)     /* R19: trace horizon bound */
+#define CONVGPU_NONE32 0xFFFFFFFFu        /* admit_tick of a never-admitted container */
+#define CONVGPU_NONE8 0xFFu               /* admit_rank of a never-admitted container */
+
+/* The four scheduling policies of P:141-145 (R3-R7). */
+typedef enum {
+  CONVGPU_FIFO = 0,        /* oldest created paused container */
+  CONVGPU_BEST_FIT = 1,    /* shortfall closest to, not above, free memory */
+  CONVGPU_RECENT_FIT = 2,  /* most recently suspended ("Recent use") */
+  CONVGPU_RANDOM_FIT = 3   /* uniform among paused ("Random"), Philox-keyed */
+} convgpu_policy_t;
+
+/* Op kinds: op_arg = kind << 30 | size_mib (size < 2^30).  The replay maps
+ * the wrapper-module API classes of Table II: allocation APIs ->
+ * ALLOC, cudaFree -> FREE, __cudaUnregisterFatBinary /
+ * container stop -> FINISH; NOP = compute without memory calls. */
+typedef enum {
+  CONVGPU_OP_ALLOC = 0,
+  CONVGPU_OP_FREE = 1,
+  CONVGPU_OP_FINISH = 2,
+  CONVGPU_OP_NOP = 3
+} convgpu_op_t;
+
+/* Per-trace flag bits (summary.flags, stats.flag_count[bit]).  Bit 1 is an
+ * assertion and does not stop the trace; any other bit stops it, its
+ * per-container outputs become (NONE32, NONE8, 0, 0) and every summary field
+ * except flags is 0. */
+enum {
+  CONVGPU_FLAG_DEADLOCK = 1u << 0,         /* containers remain, none can run (P:7) */
+  CONVGPU_FLAG_OVERCOMMIT = 1u << 1,       /* memory in use > memory reserved */
+  CONVGPU_FLAG_INVALID_LIMIT = 1u << 2,    /* a declared limit > capacity (R15) */
+  CONVGPU_FLAG_INVALID_FREE = 1u << 3,     /* FREE of more than the container uses */
+  CONVGPU_FLAG_UNSORTED_ARRIVAL = 1u << 4, /* arrival[c] < arrival[c-1] */
+  CONVGPU_FLAG_TICK_RANGE = 1u << 5,       /* max arrival + sum of deltas >= 2^26 */
+  CONVGPU_FLAG_BAD_PROGRAM = 1u << 6       /* last op not FINISH or FINISH not last */
+};
+
+/* A batch of n independent traces, structure-of-arrays in DEVICE memory.
+ * Trace i, container c (0 <= c < n_containers), op k (0 <= k < n_ops):
+ *   arrival[i*n_containers + c]                 tick of container creation
+ *   limit[i*n_containers + c]                   declared GPU-memory limit, MiB
+ *   op_delta[(i*n_ops + k)*n_containers + c]    ticks after the previous op
+ *                                               (after arrival for k = 0)
+ *   op_arg[(i*n_ops + k)*n_containers + c]      kind << 30 | size_mib
+ * Arrivals must be non-decreasing within a trace (index = creation order,
+ * R7) and every container's last op must be its only FINISH.
+ * Fastest path: n_containers % 4 == 0 and 16-byte aligned arrays (traces are
+ * then staged into shared memory by the bulk-copy engine). */
+typedef struct {
+  const uint32_t *arrival, *limit, *op_delta, *op_arg; /* device */
+  uint32_t n_containers;     /* 1..64 */
+  uint32_t n_ops;            /* K, 1..8 */
+  uint64_t trace_id_base;    /* global id of trace 0 (sharding; Random-Fit counter) */
+  uint64_t rand_seed;        /* Random-Fit Philox key (R6) */
+  uint32_t ctx_overhead_mib; /* charged at a container's first ALLOC (66) */
+  uint32_t reserved0;        /* must be 0 */
+} convgpu_traces_t;
+
+/* Per-trace summary, 40 bytes. */
+typedef struct {
+  uint32_t makespan;      /* max finish - arrival[0] (Table IV "finished time") */
+  uint32_t peak_reserved; /* max over events of capacity - free */
+  uint32_t peak_used;     /* max over events of sum of used */
+  uint32_t flags;         /* CONVGPU_FLAG_* */
+  uint64_t sum_wait;      /* total suspended ticks (Table V numerator) */
+  uint32_t n_rejected;    /* ALLOCs denied for exceeding the limit */
+  uint32_t n_select;      /* policy selections made */
+  uint64_t digest;        /* DESIGN.md R20 digest of all outputs of the trace */
+} convgpu_summary_t;
+
+/* Batch statistics, accumulated with device atomics into caller-zeroed
+ * DEVICE memory (several calls may accumulate into one struct). */
+typedef struct {
+  uint64_t traces, events, sum_makespan, sum_wait, n_rejected, n_select, digest_sum;
+  uint32_t max_makespan, max_peak_reserved;
+  uint32_t flag_count[8];
+} convgpu_stats_t;
+
+/* Outputs; every pointer is DEVICE memory or NULL (= not produced). */
+typedef struct {
+  uint32_t *admit_tick;  /* [n][n_containers] tick the limit became fully assigned */
+  uint8_t *admit_rank;   /* [n][n_containers] admission order, NONE8 if never */
+  uint32_t *wait;        /* [n][n_containers] ticks spent suspended */
+  uint32_t *finish;      /* [n][n_containers] tick of FINISH */
+  convgpu_summary_t *summary; /* [n] */
+  convgpu_stats_t *stats;     /* 1 struct, caller-zeroed, accumulated */
+  uint64_t *range_digest;     /* optional: range_digest[gid / range_size] += digest */
+  uint64_t range_size;        /* > 0 when range_digest != NULL */
+  void *stream;               /* cudaStream_t */
+} convgpu_out_t;
+
+/*
+ * convgpu_replay — replay n traces under one policy (the hot path).
+ * Semantics: DESIGN.md §Semantics; P:78, P:98, P:104, P:110, P:133-145,
+ * P:149.  One warp per trace; the event loop, policy selection, outputs,
+ * digests and the statistics reduction all run in the kernel.
+ * capacity_mib: GPU memory to share, 1 .. CONVGPU_CAPACITY_LIMIT-1.
+ * policy: convgpu_policy_t.  n may be 0 (no-op).
+ * Errors: -EINVAL for NULL traces/out/arrays, n_containers or n_ops out of
+ * range, policy out of range, capacity out of range, overhead out of range,
+ * reserved0 != 0, host pointers, range_digest without range_size; -ENODEV;
+ * -EIO (launch failure).
+ */
+int convgpu_replay(const convgpu_traces_t *traces, uint64_t n, uint32_t capacity_mib,
+                   int policy, const convgpu_out_t *out);
+
+/* Synthetic workload generator (DESIGN.md §Input recipe; P:179 random
+ * Table III types every 5 s, P:181-187 sizes, "5 to 45 seconds" by size).
+ * Per trace id g and container c, Philox4x32-10 with counter
+ * (lo32 g, hi32 g, c, 0) and key gen_seed gives (x0, x1):
+ *   k = (x0 * n_classes) >> 32, L = class_mib[k] * num / den,
+ *   arrival = c * iat, dur = dur_base + dur_step * (k + dur_class_offset)
+ *         + ((x1 * (dur_jit + 1)) >> 32), e = max(L - ovh, 0);
+ *   n_ops = 4: ALLOC e/2 @0, ALLOC e - e/2 @dur/4, FREE e/2 @dur/2,
+ *              FINISH @dur - dur/4 - dur/2;
+ *   n_ops = 2: ALLOC e @0, FINISH @dur (paper-mimic). */
+typedef struct {
+  uint64_t gen_seed;
+  uint32_t n_containers, n_ops;  /* 1..64; 4 or 2 */
+  uint32_t n_classes;            /* 1..8 */
+  uint32_t class_mib[8];
+  uint32_t num, den;             /* den > 0 */
+  uint32_t iat;
+  uint32_t dur_base, dur_step, dur_class_offset, dur_jit;
+  uint32_t ctx_overhead_mib;
+} convgpu_gen_params_t;
+
+/* Writable DEVICE buffers for convgpu_generate, same layout as
+ * convgpu_traces_t for the generated trace ids [trace_id_base, +n). */
+typedef struct {
+  uint32_t *arrival, *limit, *op_delta, *op_arg;
+} convgpu_trace_buffers_t;
+
+/* Generate n traces with global ids trace_id_base .. +n-1 into dst.
+ * Errors: -EINVAL (NULL, bad params, host pointers), -ENODEV, -EIO. */
+int convgpu_generate(const convgpu_gen_params_t *params, uint64_t trace_id_base,
+                     uint64_t n, const convgpu_trace_buffers_t *dst, void *stream);
+
+/* End-to-end replay from HOST memory (pinned for full speed): traces->arrays
+ * are HOST pointers.  The batch is streamed through the caller's DEVICE
+ * workspace in chunks of chunk_traces traces; the copy-in of chunk j+1 (on an
+ * internal stream) overlaps the replay of chunk j (on `stream`), and every
+ * policy whose bit is set in policy_mask (bit q = convgpu_policy_t q) is
+ * replayed on the chunk while it is resident.  Outputs go back to HOST:
+ *   host_summary: [n_policies][n] records (NULL = not produced),
+ *   host_stats:   [n_policies] records, overwritten (not accumulated),
+ * in increasing policy order.  workspace: DEVICE, at least
+ * convgpu_replay_host_workspace(n_containers, n_ops, chunk_traces,
+ * n_policies) bytes.  Synchronous: returns when the results are in host
+ * memory; all work is joined into `stream`, so CUDA events recorded on
+ * `stream` around the call bracket every copy and kernel.
+ * Errors: -EINVAL (bad shape, empty mask, small workspace, host workspace),
+ * -ENODEV, -EIO. */
+size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops,
+                                     uint64_t chunk_traces, uint32_t n_policies);
+int convgpu_replay_host(const convgpu_traces_t *host_traces, uint64_t n,
+                        uint32_t capacity_mib, uint32_t policy_mask,
+                        convgpu_summary_t *host_summary, convgpu_stats_t *host_stats,
+                        void *device_workspace, size_t workspace_bytes,
+                        uint64_t chunk_traces, void *stream);
+
+/* Number of kernel launches convgpu_replay and convgpu_generate enqueue per
+ * call (convgpu_replay_host: this many per chunk and policy). */
+int convgpu_launches_per_call(void);
+
+/* Human-readable text for a return code (thread-local CUDA text for -EIO). */
+const char *convgpu_strerror(int rc);
+
+/* CONVGPU_ABI_VERSION of the loaded library. */
+int convgpu_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CONVGPU_H */

@@ -1,0 +1,258 @@
+// abi.cu — the extern "C" boundary of libconvgpu.so (include/convgpu.h):
+// argument validation, device check, error mapping, launch configuration and
+// the chunked host-memory end-to-end path.  Every computation runs in the
+// kernels of replay.cu / generate.cu.
+#include <cuda_runtime.h>
+#include <errno.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+
+#include "convgpu.h"
+#include "internal.h"
+
+namespace {
+
+thread_local char g_err[256];
+
+int fail_cuda(cudaError_t e, const char* where) {
+  snprintf(g_err, sizeof g_err, "%s: %s (%s)", where, cudaGetErrorString(e), cudaGetErrorName(e));
+  cudaGetLastError();  // clear sticky-free errors
+  return -EIO;
+}
+
+int check_device() {
+  int dev = 0, major = 0, minor = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e == cudaErrorNoDevice ? -ENODEV : fail_cuda(e, "cudaGetDevice");
+  if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev) != cudaSuccess)
+    return -ENODEV;
+  if (major != 10 || minor != 0) return -ENODEV;  // built for sm_100a only
+  return 0;
+}
+
+// Device (or managed) memory on the current device.
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+bool opt_device_ptr(const void* p) { return p == nullptr || is_device_ptr(p); }
+
+bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
+  if (!t) return -EINVAL;
+  if (t->n_containers < 1 || t->n_containers > CONVGPU_MAX_CONTAINERS) return -EINVAL;
+  if (t->n_ops < 1 || t->n_ops > CONVGPU_MAX_OPS) return -EINVAL;
+  if (policy < 0 || policy > 3) return -EINVAL;
+  if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
+  if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
+  if (t->reserved0 != 0) return -EINVAL;
+  return 0;
+}
+
+int validate_arrays(const convgpu_traces_t* t) {
+  if (!t->arrival || !t->limit || !t->op_delta || !t->op_arg) return -EINVAL;
+  return 0;
+}
+
+convgpu::ReplayArgs make_args(const convgpu_traces_t* t, uint64_t n, uint32_t cap) {
+  convgpu::ReplayArgs a;
+  memset(&a, 0, sizeof a);
+  a.arrival = t->arrival; a.limit = t->limit; a.delta = t->op_delta; a.arg = t->op_arg;
+  a.n = t->n_containers; a.K = t->n_ops;
+  a.tid_base = t->trace_id_base; a.seed = t->rand_seed;
+  a.ovh = t->ctx_overhead_mib; a.cap = cap; a.count = n;
+  return a;
+}
+
+bool use_bulk(const convgpu::ReplayArgs& a) {
+  return (a.n % 4u) == 0 && aligned16(a.arrival) && aligned16(a.limit) && aligned16(a.delta) &&
+         aligned16(a.arg);
+}
+
+}  // namespace
+
+extern "C" {
+
+int convgpu_abi_version(void) { return CONVGPU_ABI_VERSION; }
+
+int convgpu_launches_per_call(void) { return 1; }
+
+const char* convgpu_strerror(int rc) {
+  switch (rc) {
+    case 0: return "success";
+    case -EINVAL: return "invalid argument (see include/convgpu.h)";
+    case -ENODEV: return "no sm_100 (B200-class) CUDA device is current";
+    case -EIO: return g_err[0] ? g_err : "CUDA error";
+    default: return "unknown error";
+  }
+}
+
+int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity_mib, int policy,
+                   const convgpu_out_t* out) {
+  int rc = validate_shape(traces, capacity_mib, policy);
+  if (rc) return rc;
+  if (!out) return -EINVAL;
+  if (out->range_digest && out->range_size == 0) return -EINVAL;
+  if (n == 0) return 0;  // no-op: array pointers may be NULL
+  if ((rc = validate_arrays(traces))) return rc;
+  if ((rc = check_device())) return rc;
+  if (!is_device_ptr(traces->arrival) || !is_device_ptr(traces->limit) ||
+      !is_device_ptr(traces->op_delta) || !is_device_ptr(traces->op_arg))
+    return -EINVAL;
+  if (!opt_device_ptr(out->admit_tick) || !opt_device_ptr(out->admit_rank) ||
+      !opt_device_ptr(out->wait) || !opt_device_ptr(out->finish) ||
+      !opt_device_ptr(out->summary) || !opt_device_ptr(out->stats) ||
+      !opt_device_ptr(out->range_digest))
+    return -EINVAL;
+  convgpu::ReplayArgs a = make_args(traces, n, capacity_mib);
+  a.admit_tick = out->admit_tick; a.admit_rank = out->admit_rank;
+  a.wait = out->wait; a.finish = out->finish;
+  a.summary = out->summary; a.stats = out->stats;
+  a.range_digest = out->range_digest; a.range_size = out->range_size;
+  cudaError_t e = convgpu::launch_replay(a, policy, use_bulk(a), (cudaStream_t)out->stream);
+  return e == cudaSuccess ? 0 : fail_cuda(e, "replay launch");
+}
+
+int convgpu_generate(const convgpu_gen_params_t* p, uint64_t trace_id_base, uint64_t n,
+                     const convgpu_trace_buffers_t* dst, void* stream) {
+  if (!p || !dst) return -EINVAL;
+  if (p->n_containers < 1 || p->n_containers > CONVGPU_MAX_CONTAINERS) return -EINVAL;
+  if (p->n_ops != 4 && p->n_ops != 2) return -EINVAL;
+  if (p->n_classes < 1 || p->n_classes > 8 || p->den == 0) return -EINVAL;
+  int rc = check_device();
+  if (rc) return rc;
+  if (n == 0) return 0;
+  if (!is_device_ptr(dst->arrival) || !is_device_ptr(dst->limit) || !is_device_ptr(dst->op_delta) ||
+      !is_device_ptr(dst->op_arg))
+    return -EINVAL;
+  convgpu::GenArgs a;
+  a.p = *p; a.tid_base = trace_id_base; a.count = n;
+  a.arrival = dst->arrival; a.limit = dst->limit; a.delta = dst->op_delta; a.arg = dst->op_arg;
+  cudaError_t e = convgpu::launch_generate(a, (cudaStream_t)stream);
+  return e == cudaSuccess ? 0 : fail_cuda(e, "generate launch");
+}
+
+// ---------------------------------------------------------------- host e2e
+// Workspace layout (256-B aligned pieces): 2 x {arrival, limit, delta, arg}
+// chunk buffers, 2 x n_policies summary chunks, n_policies stats structs.
+static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops, uint64_t chunk,
+                                     uint32_t n_policies) {
+  const size_t cn = align256(chunk * n_containers * 4);
+  const size_t ckn = align256(chunk * n_containers * n_ops * 4);
+  return 2 * (2 * cn + 2 * ckn) + 2 * (size_t)n_policies * align256(chunk * sizeof(convgpu_summary_t)) +
+         (size_t)n_policies * align256(sizeof(convgpu_stats_t));
+}
+
+int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, uint32_t policy_mask,
+                        convgpu_summary_t* host_summary, convgpu_stats_t* host_stats,
+                        void* ws, size_t ws_bytes, uint64_t chunk, void* stream_) {
+  if (policy_mask == 0 || policy_mask > 0xFu) return -EINVAL;
+  int rc = validate_shape(ht, cap, 0);
+  if (rc) return rc;
+  if (!host_stats || !ws || chunk == 0) return -EINVAL;
+  if ((rc = validate_arrays(ht))) return rc;
+  if ((rc = check_device())) return rc;
+  int pols[4], np = 0;
+  for (int q = 0; q < 4; ++q)
+    if (policy_mask & (1u << q)) pols[np++] = q;
+  const uint32_t nc = ht->n_containers, K = ht->n_ops;
+  if (ws_bytes < convgpu_replay_host_workspace(nc, K, chunk, (uint32_t)np) || !is_device_ptr(ws))
+    return -EINVAL;
+  cudaStream_t cs = (cudaStream_t)stream_;
+  const size_t cn = align256(chunk * nc * 4), ckn = align256(chunk * nc * K * 4);
+  const size_t sb = align256(chunk * sizeof(convgpu_summary_t));
+  char* w = (char*)ws;
+  uint32_t *arr[2], *lim[2], *del[2], *arg[2];
+  convgpu_summary_t* sum[2][4];
+  for (int b = 0; b < 2; ++b) {
+    arr[b] = (uint32_t*)w; w += cn;
+    lim[b] = (uint32_t*)w; w += cn;
+    del[b] = (uint32_t*)w; w += ckn;
+    arg[b] = (uint32_t*)w; w += ckn;
+  }
+  for (int b = 0; b < 2; ++b)
+    for (int q = 0; q < np; ++q) { sum[b][q] = (convgpu_summary_t*)w; w += sb; }
+  convgpu_stats_t* dstats = (convgpu_stats_t*)w;  // [np], 256-B apart
+  const size_t stb = align256(sizeof(convgpu_stats_t));
+
+  cudaStream_t copy = nullptr;
+  cudaEvent_t h2d[2] = {nullptr, nullptr}, kdone[2] = {nullptr, nullptr};
+  cudaEvent_t start_ev = nullptr, copy_done = nullptr;
+  cudaError_t e = cudaStreamCreateWithFlags(&copy, cudaStreamNonBlocking);
+  for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
+    e = cudaEventCreateWithFlags(&h2d[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&kdone[b], cudaEventDisableTiming);
+  }
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&copy_done, cudaEventDisableTiming);
+  const uint64_t nchunks = (n + chunk - 1) / chunk;
+  auto enqueue_h2d = [&](uint64_t j) -> cudaError_t {
+    const int b = (int)(j & 1);
+    const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
+    cudaError_t r = cudaSuccess;
+    if (j >= 2) r = cudaStreamWaitEvent(copy, kdone[b], 0);  // buffer b free again
+    if (r == cudaSuccess) r = cudaMemcpyAsync(arr[b], ht->arrival + lo * nc, cnt * nc * 4, cudaMemcpyHostToDevice, copy);
+    if (r == cudaSuccess) r = cudaMemcpyAsync(lim[b], ht->limit + lo * nc, cnt * nc * 4, cudaMemcpyHostToDevice, copy);
+    if (r == cudaSuccess) r = cudaMemcpyAsync(del[b], ht->op_delta + lo * nc * K, cnt * nc * K * 4, cudaMemcpyHostToDevice, copy);
+    if (r == cudaSuccess) r = cudaMemcpyAsync(arg[b], ht->op_arg + lo * nc * K, cnt * nc * K * 4, cudaMemcpyHostToDevice, copy);
+    if (r == cudaSuccess) r = cudaEventRecord(h2d[b], copy);
+    return r;
+  };
+  for (int q = 0; q < np && e == cudaSuccess; ++q)
+    e = cudaMemsetAsync((char*)dstats + q * stb, 0, sizeof(convgpu_stats_t), cs);
+  if (e == cudaSuccess) e = cudaEventRecord(start_ev, cs);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(copy, start_ev, 0);
+  if (e == cudaSuccess && nchunks) e = enqueue_h2d(0);
+  for (uint64_t j = 0; j < nchunks && e == cudaSuccess; ++j) {
+    const int b = (int)(j & 1);
+    const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
+    if (j + 1 < nchunks) e = enqueue_h2d(j + 1);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, h2d[b], 0);
+    if (e != cudaSuccess) break;
+    convgpu_traces_t dt = *ht;
+    dt.arrival = arr[b]; dt.limit = lim[b]; dt.op_delta = del[b]; dt.op_arg = arg[b];
+    dt.trace_id_base = ht->trace_id_base + lo;
+    for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
+      convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
+      a.summary = host_summary ? sum[b][q] : nullptr;
+      a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
+      e = convgpu::launch_replay(a, pols[q], use_bulk(a), cs);
+    }
+    if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
+    if (e == cudaSuccess && host_summary) {
+      e = cudaStreamWaitEvent(copy, kdone[b], 0);
+      for (int q = 0; q < np && e == cudaSuccess; ++q)
+        e = cudaMemcpyAsync(host_summary + (uint64_t)q * n + lo, sum[b][q],
+                            cnt * sizeof(convgpu_summary_t), cudaMemcpyDeviceToHost, copy);
+    }
+  }
+  for (int q = 0; q < np && e == cudaSuccess; ++q)
+    e = cudaMemcpyAsync(host_stats + q, (char*)dstats + q * stb, sizeof(convgpu_stats_t),
+                        cudaMemcpyDeviceToHost, cs);
+  // join the copy stream back into the caller's stream (events on `stream`
+  // then bracket every copy and kernel of the call)
+  if (e == cudaSuccess) e = cudaEventRecord(copy_done, copy);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, copy_done, 0);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+  for (int b = 0; b < 2; ++b) {
+    if (h2d[b]) cudaEventDestroy(h2d[b]);
+    if (kdone[b]) cudaEventDestroy(kdone[b]);
+  }
+  if (start_ev) cudaEventDestroy(start_ev);
+  if (copy_done) cudaEventDestroy(copy_done);
+  if (copy) cudaStreamDestroy(copy);
+  return e == cudaSuccess ? 0 : fail_cuda(e, "replay_host");
+}
+
+}  // extern "C"

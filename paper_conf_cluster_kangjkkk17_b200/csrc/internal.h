@@ -1,0 +1,39 @@
+// internal.h — launch structs shared by the CUDA translation units of
+// libconvgpu.so (not part of the public ABI; see include/convgpu.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "convgpu.h"
+
+namespace convgpu {
+
+constexpr int kReplayThreads = 128;  // 4 warps, one trace each at a time
+
+struct ReplayArgs {
+  const uint32_t *arrival, *limit, *delta, *arg;
+  uint32_t n, K;
+  uint64_t tid_base, seed;
+  uint32_t ovh, cap;
+  uint64_t count;
+  uint32_t* admit_tick;
+  uint8_t* admit_rank;
+  uint32_t *wait, *finish;
+  convgpu_summary_t* summary;
+  convgpu_stats_t* stats;
+  uint64_t* range_digest;
+  uint64_t range_size;
+  uint64_t grid_override;  // 0 = occupancy-sized persistent grid
+};
+
+cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream);
+
+struct GenArgs {
+  convgpu_gen_params_t p;
+  uint64_t tid_base, count;
+  uint32_t *arrival, *limit, *delta, *arg;
+};
+
+cudaError_t launch_generate(const GenArgs& a, cudaStream_t stream);
+
+}  // namespace convgpu

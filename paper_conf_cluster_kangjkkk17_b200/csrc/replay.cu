@@ -1,0 +1,499 @@
+// replay.cu — the hot path: batched replay of ConVGPU's GPU-memory scheduler
+// (§III-D, Fig. 3) on sm_100a.
+//
+// Design:
+//  * one warp per trace, persistent grid-stride over traces;
+//  * the next trace's SoA arrays are prefetched into a per-warp shared-memory
+//    double buffer by the bulk-copy (TMA) engine — cp.async.bulk completing
+//    on an mbarrier — while the warp replays the current trace;
+//  * event keys (tick << 6 | container) live in registers, two containers
+//    per lane; the next event is one __reduce_min_sync (redux.sync.min);
+//  * per-container ledger (used, wait, admission, op cursor, flags) lives in
+//    shared memory and is updated by warp-uniform code (broadcast reads), the
+//    scheduler ledger (free memory, fill target, counters) in uniform
+//    registers — no divergence in the event loop;
+//  * policy selection is lane-parallel: FIFO = find-first-set of
+//    the paused mask, Best-Fit = two packed redux (max fitting shortfall,
+//    else min shortfall), Recent-Fit = redux.max over packed suspension
+//    numbers, Random-Fit = Philox draw + popc + fns over the paused mask;
+//  * outputs, the R20 digest, and a warp -> block -> grid statistics
+//    reduction are fused into the trace epilogue / kernel tail.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace convgpu {
+
+// Per-container state word in shared memory.
+enum : uint32_t {
+  kStK = 0xFu,              // index of the next op
+  kStArrived = 1u << 4,
+  kStFirst = 1u << 5,       // first allocation of the pid done
+  kStAdmitted = 1u << 6,    // assignment == declared limit
+  kStPaused = 1u << 7,      // allocation reply withheld
+};
+constexpr uint32_t kTargetNone = 64u;
+constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
+constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
+
+struct WarpStats {  // 96 B, per warp, shared memory
+  unsigned long long traces, events, sum_makespan, sum_wait, n_rejected, n_select, digest_sum;
+  uint32_t max_makespan, max_peak_reserved;
+  uint32_t flag_count[8];
+};
+static_assert(sizeof(WarpStats) == 96, "WarpStats layout");
+
+constexpr uint32_t kHeaderBytes = 128;         // 2 mbarriers + WarpStats + range acc
+constexpr uint32_t kStateWords = 6 * 64;       // used, wait, admit, st, fin, seq
+
+__host__ __device__ inline uint32_t in_words(uint32_t n, uint32_t K) { return (2 + 2 * K) * n; }
+__host__ __device__ inline uint32_t warp_region_bytes(uint32_t n, uint32_t K) {
+  uint32_t b = kHeaderBytes + kStateWords * 4 + 2 * in_words(n, K) * 4;
+  return (b + 15u) & ~15u;
+}
+
+// ---------------------------------------------------------------- TMA bits
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("{\n\t.reg .b64 st;\n\tmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n\t}" ::"r"(
+                   smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+// ---------------------------------------------------------------- kernel
+template <int POLICY, bool BULK>
+__global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayArgs p) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint32_t wib = threadIdx.x >> 5;
+  const uint32_t n = p.n, K = p.K;
+  const uint32_t IN = in_words(n, K);
+  unsigned char* base = smem + wib * warp_region_bytes(n, K);
+  uint64_t* mbar = reinterpret_cast<uint64_t*>(base);
+  WarpStats* ws = reinterpret_cast<WarpStats*>(base + 16);
+  unsigned long long* racc = reinterpret_cast<unsigned long long*>(base + 112);  // [cur, acc]
+  uint32_t* s_used = reinterpret_cast<uint32_t*>(base + kHeaderBytes);
+  uint32_t* s_wait = s_used + 64;
+  uint32_t* s_admit = s_used + 128;  // tick << 6 | rank, or kKeyNone
+  uint32_t* s_st = s_used + 192;
+  uint32_t* s_fin = s_used + 256;
+  uint32_t* s_seq = s_used + 320;
+  uint32_t* inbuf = s_used + kStateWords;  // [2][IN]
+
+  const uint64_t warps_per_block = blockDim.x >> 5;
+  const uint64_t gw = (uint64_t)blockIdx.x * warps_per_block + wib;
+  const uint64_t W = (uint64_t)gridDim.x * warps_per_block;
+
+  if (lane == 0) {
+    unsigned long long* z = reinterpret_cast<unsigned long long*>(ws);
+#pragma unroll
+    for (int j = 0; j < 12; ++j) z[j] = 0ull;
+    racc[0] = ~0ull;
+    racc[1] = 0ull;
+    if (BULK) {
+      mbar_init(&mbar[0]);
+      mbar_init(&mbar[1]);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+  }
+  __syncwarp();
+
+  auto prefetch = [&](uint64_t i, uint32_t b) {
+    uint32_t* dst = inbuf + b * IN;
+    if (BULK) {
+      if (lane == 0) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        const uint32_t nb = n * 4u, knb = K * n * 4u;
+        mbar_expect_tx(&mbar[b], 2u * nb + 2u * knb);
+        bulk_g2s(dst, p.arrival + i * n, nb, &mbar[b]);
+        bulk_g2s(dst + n, p.limit + i * n, nb, &mbar[b]);
+        bulk_g2s(dst + 2 * n, p.delta + i * (uint64_t)K * n, knb, &mbar[b]);
+        bulk_g2s(dst + 2 * n + K * n, p.arg + i * (uint64_t)K * n, knb, &mbar[b]);
+      }
+    } else {
+      for (uint32_t j = lane; j < n; j += 32) {
+        dst[j] = __ldg(p.arrival + i * n + j);
+        dst[n + j] = __ldg(p.limit + i * n + j);
+      }
+      const uint64_t ob = i * (uint64_t)K * n;
+      for (uint32_t j = lane; j < K * n; j += 32) {
+        dst[2 * n + j] = __ldg(p.delta + ob + j);
+        dst[2 * n + K * n + j] = __ldg(p.arg + ob + j);
+      }
+    }
+  };
+
+  uint32_t phase = 0;  // bit b = parity to wait for on buffer b
+  if (BULK && gw < p.count) prefetch(gw, 0);
+
+  uint64_t j = 0;
+  for (uint64_t i = gw; i < p.count; i += W, ++j) {
+    const uint32_t b = (uint32_t)(j & 1);
+    if (BULK) {
+      if (i + W < p.count) prefetch(i + W, b ^ 1u);
+      mbar_wait(&mbar[b], (phase >> b) & 1u);
+      phase ^= 1u << b;
+    } else {
+      __syncwarp();
+      prefetch(i, 0);
+      __syncwarp();
+    }
+    const uint32_t* A = inbuf + (BULK ? b * IN : 0);
+    const uint32_t* Lm = A + n;
+    const uint32_t* D = A + 2 * n;
+    const uint32_t* R = A + 2 * n + K * n;
+    const uint64_t tid = p.tid_base + i;
+
+    // ---- per-trace init + static validation ----
+    uint32_t key0 = kKeyNone, key1 = kKeyNone;
+    uint32_t bad = 0, lsum = 0, lmax = 0;
+#pragma unroll
+    for (uint32_t s = 0; s < 2; ++s) {
+      const uint32_t c = lane + 32u * s;
+      s_used[c] = 0; s_wait[c] = 0; s_admit[c] = kKeyNone; s_st[c] = 0; s_fin[c] = 0; s_seq[c] = 0;
+      if (c < n) {
+        const uint32_t a = A[c];
+        if (Lm[c] > p.cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+        if (c > 0 && a < A[c - 1]) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
+        lmax = max(lmax, a);
+        for (uint32_t k = 0; k < K; ++k) {
+          lsum = min(lsum + min(D[k * n + c], kTickLimit), kTickLimit);
+          const bool fin = (R[k * n + c] >> 30) == CONVGPU_OP_FINISH;
+          if (fin != (k + 1 == K)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+        }
+        const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
+        if (s == 0) key0 = key; else key1 = key;
+      }
+    }
+    uint32_t flags = __reduce_or_sync(kFull, bad);
+    {
+      const uint32_t tot = __reduce_add_sync(kFull, lsum);
+      const uint32_t amax = __reduce_max_sync(kFull, lmax);
+      if (amax >= kTickLimit || amax + tot >= kTickLimit) flags |= CONVGPU_FLAG_TICK_RANGE;
+    }
+    __syncwarp();
+
+    // ---- uniform scheduler ledger (D4, D1 target, counters) ----
+    uint32_t free_mem = p.cap, target = kTargetNone, a_tg = 0, used_total = 0;
+    uint32_t seq = 0, rank = 0, draws = 0, n_rej = 0, n_sel = 0;
+    uint32_t peak_res = 0, peak_used = 0, live = n, events = 0;
+    uint32_t pm_lo = 0, pm_hi = 0;  // paused set (D3) as a 64-bit mask
+
+    auto set_key = [&](uint32_t c, uint32_t k) {
+      if (lane == (c & 31u)) {
+        if (c & 32u) key1 = k; else key0 = k;
+      }
+    };
+
+    if (flags == 0) {
+      for (;;) {
+        const uint32_t kmin = __reduce_min_sync(kFull, min(key0, key1));
+        if (kmin == kKeyNone) {
+          if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
+          break;
+        }
+        const uint32_t t = kmin >> 6, c = kmin & 63u;
+        ++events;
+        uint32_t st = s_st[c];
+        const uint32_t L = Lm[c];
+        uint32_t nk = kKeyNone;
+        bool disp = false;
+        if (!(st & kStArrived)) {
+          // ARRIVE (Fig. 3b/3c; R2)
+          const uint32_t g = (target == kTargetNone) ? min(L, free_mem) : 0u;
+          free_mem -= g;
+          st |= kStArrived;
+          if (g == L) {
+            s_admit[c] = (t << 6) | rank; ++rank; st |= kStAdmitted;
+          } else if (g > 0) {
+            target = c; a_tg = g;
+          }
+          nk = ((t + D[c]) << 6) | c;
+        } else {
+          uint32_t k = st & kStK;
+          const uint32_t w = R[k * n + c];
+          const uint32_t kind = w >> 30, r = w & kSizeMask;
+          bool adv = true;
+          if (kind == CONVGPU_OP_ALLOC) {
+            const uint32_t used = s_used[c];
+            const uint32_t need = used + r + ((st & kStFirst) ? 0u : p.ovh);
+            const uint32_t a = (st & kStAdmitted) ? L : (c == target ? a_tg : 0u);
+            if (need > L) {
+              ++n_rej;  // R10
+            } else if (need <= a) {
+              s_used[c] = need; used_total += need - used; st |= kStFirst;
+            } else {  // pause: reply withheld
+              st |= kStPaused;
+              s_wait[c] -= t;
+              if (POLICY == CONVGPU_RECENT_FIT) s_seq[c] = seq;
+              ++seq;
+              if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
+              adv = false;
+              disp = (target == kTargetNone);
+            }
+          } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
+            const uint32_t used = s_used[c];
+            if (r > used) { flags |= CONVGPU_FLAG_INVALID_FREE; break; }
+            s_used[c] = used - r; used_total -= r;
+          } else if (kind == CONVGPU_OP_FINISH) {  // P:110, R18
+            const uint32_t a = (st & kStAdmitted) ? L : (c == target ? a_tg : 0u);
+            free_mem += a;
+            used_total -= s_used[c];
+            s_used[c] = 0;
+            s_fin[c] = t;
+            --live;
+            if (c == target) { target = kTargetNone; a_tg = 0; }  // R20
+            adv = false;
+            disp = true;
+          }
+          if (adv) {
+            ++k;
+            st = (st & ~kStK) | k;
+            nk = ((t + D[k * n + c]) << 6) | c;
+          }
+        }
+        s_st[c] = st;
+        set_key(c, nk);
+
+        // ---- DISPATCH (Fig. 3d; R1, R9) ----
+        if (disp) {
+          for (;;) {
+            if (target != kTargetNone) {
+              const uint32_t tg = target, Lt = Lm[tg];
+              const uint32_t g = min(free_mem, Lt - a_tg);
+              a_tg += g;
+              free_mem -= g;
+              uint32_t stt = s_st[tg];
+              if (stt & kStPaused) {
+                uint32_t kt = stt & kStK;
+                const uint32_t pend = (R[kt * n + tg] & kSizeMask) + ((stt & kStFirst) ? 0u : p.ovh);
+                const uint32_t ut = s_used[tg];
+                if (ut + pend <= a_tg) {  // RESUME (R9)
+                  s_used[tg] = ut + pend;
+                  used_total += pend;
+                  s_wait[tg] += t;
+                  if (tg < 32) pm_lo &= ~(1u << tg); else pm_hi &= ~(1u << (tg - 32));
+                  ++kt;
+                  stt = (stt & ~(kStK | kStPaused)) | kStFirst | kt;
+                  set_key(tg, ((t + D[kt * n + tg]) << 6) | tg);
+                }
+              }
+              if (a_tg == Lt) {  // fully guaranteed: admit, cascade leftover
+                s_admit[tg] = (t << 6) | rank; ++rank;
+                s_st[tg] = stt | kStAdmitted;
+                target = kTargetNone;
+                a_tg = 0;
+                continue;
+              }
+              s_st[tg] = stt;
+              break;
+            }
+            if ((pm_lo | pm_hi) == 0u) break;
+            // ---- SELECT among paused ----
+            uint32_t sel;
+            if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
+              sel = pm_lo ? (uint32_t)(__ffs(pm_lo) - 1) : 32u + (uint32_t)(__ffs(pm_hi) - 1);
+            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4
+              uint32_t vf = 0, vm = kKeyNone;
+#pragma unroll
+              for (uint32_t s = 0; s < 2; ++s) {
+                const uint32_t c2 = lane + 32u * s;
+                const uint32_t m = s ? pm_hi : pm_lo;
+                if ((m >> lane) & 1u) {
+                  const uint32_t need = Lm[c2];  // shortfall L - a, a = 0 when selectable
+                  if (need <= free_mem) vf = max(vf, (need << 6) | (63u - c2));
+                  vm = min(vm, (need << 6) | c2);
+                }
+              }
+              const uint32_t kf = __reduce_max_sync(kFull, vf);
+              if (kf) {
+                sel = 63u - (kf & 63u);
+              } else {
+                sel = __reduce_min_sync(kFull, vm) & 63u;
+              }
+            } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
+              uint32_t v = 0;
+              if ((pm_lo >> lane) & 1u) v = ((s_seq[lane] + 1u) << 6) | lane;
+              if ((pm_hi >> lane) & 1u) v = max(v, ((s_seq[lane + 32] + 1u) << 6) | (lane + 32u));
+              sel = __reduce_max_sync(kFull, v) & 63u;
+            } else {  // RANDOM_FIT (R6)
+              const uint32_t clo = __popc(pm_lo);
+              const uint32_t m = clo + __popc(pm_hi);
+              const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                         (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+              ++draws;
+              const uint32_t jj = __umulhi(x.x, m);
+              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+            }
+            target = sel;
+            a_tg = 0;
+            ++n_sel;
+          }
+        }
+        const uint32_t reserved = p.cap - free_mem;
+        peak_res = max(peak_res, reserved);
+        peak_used = max(peak_used, used_total);
+        if (free_mem > p.cap || used_total > reserved) flags |= CONVGPU_FLAG_OVERCOMMIT;
+      }
+    }
+
+    // ---- epilogue: outputs, digest (R20), statistics ----
+    const bool stopped = (flags & kStopMask) != 0;
+    if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
+    uint64_t dig = 0;
+    uint32_t mfin = 0, wlo = 0, whi = 0;
+#pragma unroll
+    for (uint32_t s = 0; s < 2; ++s) {
+      const uint32_t c = lane + 32u * s;
+      if (c < n) {
+        uint32_t at = kKeyNone, ar = 0xFFu, wt = 0, fn = 0;
+        if (!stopped) {
+          const uint32_t adm = s_admit[c];
+          if (adm != kKeyNone) { at = adm >> 6; ar = adm & 63u; }
+          wt = s_wait[c];
+          fn = s_fin[c];
+        }
+        const uint64_t gi = i * n + c;
+        if (p.admit_tick) p.admit_tick[gi] = at;
+        if (p.admit_rank) p.admit_rank[gi] = (uint8_t)ar;
+        if (p.wait) p.wait[gi] = wt;
+        if (p.finish) p.finish[gi] = fn;
+        const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar << 48) ^ (uint64_t)at);
+        dig += mix64(h1 ^ (((uint64_t)wt << 32) | fn));
+        mfin = max(mfin, fn);
+        wlo += wt & 0xFFFFu;
+        whi += wt >> 16;
+      }
+    }
+    dig = warp_sum_u64(dig);
+    mfin = __reduce_max_sync(kFull, mfin);
+    const uint64_t sum_wait =
+        ((uint64_t)__reduce_add_sync(kFull, whi) << 16) + (uint64_t)__reduce_add_sync(kFull, wlo);
+    const uint32_t makespan = stopped ? 0u : mfin - A[0];
+    if (lane == 0) {
+      dig += mix64(((uint64_t)makespan << 32) | peak_res);
+      dig += mix64(((uint64_t)peak_used << 32) | flags);
+      dig += mix64(sum_wait);
+      dig += mix64(((uint64_t)n_rej << 32) | n_sel);
+      if (p.summary) {
+        convgpu_summary_t sm;
+        sm.makespan = makespan; sm.peak_reserved = peak_res; sm.peak_used = peak_used;
+        sm.flags = flags; sm.sum_wait = sum_wait; sm.n_rejected = n_rej; sm.n_select = n_sel;
+        sm.digest = dig;
+        p.summary[i] = sm;
+      }
+      ws->traces += 1; ws->events += events; ws->sum_makespan += makespan;
+      ws->sum_wait += sum_wait; ws->n_rejected += n_rej; ws->n_select += n_sel;
+      ws->digest_sum += dig;
+      ws->max_makespan = max(ws->max_makespan, makespan);
+      ws->max_peak_reserved = max(ws->max_peak_reserved, peak_res);
+      for (int bit = 0; bit < 8; ++bit) ws->flag_count[bit] += (flags >> bit) & 1u;
+      if (p.range_digest) {
+        const unsigned long long r = tid / p.range_size;
+        if (r != racc[0]) {
+          if (racc[0] != ~0ull) atomicAdd((unsigned long long*)&p.range_digest[racc[0]], racc[1]);
+          racc[0] = r;
+          racc[1] = 0;
+        }
+        racc[1] += dig;
+      }
+    }
+    __syncwarp();
+  }
+
+  // ---- tail: flush range digest, block -> grid statistics ----
+  if (lane == 0 && p.range_digest && racc[0] != ~0ull)
+    atomicAdd((unsigned long long*)&p.range_digest[racc[0]], racc[1]);
+  __syncthreads();
+  if (threadIdx.x == 0 && p.stats) {
+    WarpStats tot = *reinterpret_cast<WarpStats*>(smem + 16);
+    const uint32_t rb = warp_region_bytes(n, K);
+    for (uint32_t w = 1; w < warps_per_block; ++w) {
+      const WarpStats* o = reinterpret_cast<const WarpStats*>(smem + w * rb + 16);
+      tot.traces += o->traces; tot.events += o->events; tot.sum_makespan += o->sum_makespan;
+      tot.sum_wait += o->sum_wait; tot.n_rejected += o->n_rejected; tot.n_select += o->n_select;
+      tot.digest_sum += o->digest_sum;
+      tot.max_makespan = max(tot.max_makespan, o->max_makespan);
+      tot.max_peak_reserved = max(tot.max_peak_reserved, o->max_peak_reserved);
+      for (int bit = 0; bit < 8; ++bit) tot.flag_count[bit] += o->flag_count[bit];
+    }
+    if (tot.traces) {
+      convgpu_stats_t* S = p.stats;
+      atomicAdd((unsigned long long*)&S->traces, tot.traces);
+      atomicAdd((unsigned long long*)&S->events, tot.events);
+      atomicAdd((unsigned long long*)&S->sum_makespan, tot.sum_makespan);
+      atomicAdd((unsigned long long*)&S->sum_wait, tot.sum_wait);
+      atomicAdd((unsigned long long*)&S->n_rejected, tot.n_rejected);
+      atomicAdd((unsigned long long*)&S->n_select, tot.n_select);
+      atomicAdd((unsigned long long*)&S->digest_sum, tot.digest_sum);
+      atomicMax(&S->max_makespan, tot.max_makespan);
+      atomicMax(&S->max_peak_reserved, tot.max_peak_reserved);
+      for (int bit = 0; bit < 8; ++bit)
+        if (tot.flag_count[bit]) atomicAdd(&S->flag_count[bit], tot.flag_count[bit]);
+    }
+  }
+}
+
+// ---------------------------------------------------------------- launcher
+template <int POLICY, bool BULK>
+static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
+  const uint32_t warps = kReplayThreads / 32;
+  const size_t smem = (size_t)warps * warp_region_bytes(a.n, a.K);
+  auto kern = replay_kernel<POLICY, BULK>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 0, per_sm = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kReplayThreads, smem)) !=
+      cudaSuccess)
+    return e;
+  if (per_sm < 1) per_sm = 1;
+  const uint64_t need = (a.count + warps - 1) / warps;
+  uint64_t grid = (uint64_t)sms * (uint64_t)per_sm;
+  if (a.grid_override) grid = a.grid_override;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  kern<<<(unsigned)grid, kReplayThreads, smem, stream>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream) {
+  switch (policy * 2 + (bulk ? 1 : 0)) {
+    case 0: return launch_t<CONVGPU_FIFO, false>(a, stream);
+    case 1: return launch_t<CONVGPU_FIFO, true>(a, stream);
+    case 2: return launch_t<CONVGPU_BEST_FIT, false>(a, stream);
+    case 3: return launch_t<CONVGPU_BEST_FIT, true>(a, stream);
+    case 4: return launch_t<CONVGPU_RECENT_FIT, false>(a, stream);
+    case 5: return launch_t<CONVGPU_RECENT_FIT, true>(a, stream);
+    case 6: return launch_t<CONVGPU_RANDOM_FIT, false>(a, stream);
+    case 7: return launch_t<CONVGPU_RANDOM_FIT, true>(a, stream);
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace convgpu
