@@ -47,6 +47,7 @@ def parse():
     ap.add_argument("--workload", default="c2", choices=["c1", "c2", "mimic"])
     ap.add_argument("--traces", type=int, default=None, help="traces per GPU (default: config)")
     ap.add_argument("--outputs", default="full", choices=["full", "summary"])
+    ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -231,7 +232,8 @@ def run_ours(args, rank, local_rank, world):
             o.stats = stats[p][s]
             if timed_idx is not None:
                 ev_s[p][timed_idx].record(stream)
-            cg.replay(tr, w.cap, p, o, rand_seed=w.rand_seed, ovh=w.ovh, stream=stream)
+            cg.replay(tr, w.cap, p, o, rand_seed=w.rand_seed, ovh=w.ovh, stream=stream,
+                      kernel=args.kernel)
             if timed_idx is not None:
                 ev_e[p][timed_idx].record(stream)
             if world > 1:
@@ -262,6 +264,13 @@ def run_ours(args, rank, local_rank, world):
     ms = cgd.max_over_ranks(ms_local, dev)
 
     per_trace_events = n * (1 + K)
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+
+    def kernel_of(p):  # the rule of abi.cu auto_variant
+        if args.kernel != "auto":
+            return args.kernel
+        return "lane" if Nr >= sms * 2 * 64 * 4 and p in ("fifo", "random_fit") else "warp"
+    kernel_used = ",".join(sorted({kernel_of(p) for p in POLICIES}))
     # correctness of the timed work: every timed launch replayed every trace
     last = args.warmup + args.steps - 1
     checks = {}
@@ -286,7 +295,9 @@ def run_ours(args, rank, local_rank, world):
     achieved = bytes_per_launch / avg_launch_s / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": traffic_from_profiles(w.name, Nr),
-                "kernel": "convgpu::replay_kernel", "algorithmic_bytes_per_launch": bytes_per_launch,
+                "kernel": "replay kernels: " + ", ".join(
+                    f"{p}={kernel_of(p)}" for p in POLICIES),
+                "algorithmic_bytes_per_launch": bytes_per_launch,
                 "bytes_per_event": (in_b + out_b) / per_trace_events, "peak_source": peak_src,
                 "avg_launch_ms": avg_launch_s * 1e3,
                 "note": "issue/latency-bound warp-serial event loop; see DESIGN.md §Roofline"}
@@ -305,7 +316,7 @@ def run_ours(args, rank, local_rank, world):
                        "l2": "inputs %.2f GB per rank > 126 MB L2; no flush" % (Nr * in_b / 1e9),
                        "parallelism": f"dp{world} (trace-id shards, NCCL stats all-reduce)"},
             "per_policy": {p: {"events_per_s": Nr * per_trace_events * world / (launch_ms[p] / 1e3),
-                               "launch_ms": launch_ms[p],
+                               "launch_ms": launch_ms[p], "kernel": kernel_of(p),
                                "digest_sum": "%016x" % (checks[p]["digest_sum"] & (2**64 - 1)),
                                "sum_wait": checks[p]["sum_wait"],
                                "sum_makespan": checks[p]["sum_makespan"]} for p in POLICIES},
@@ -339,7 +350,8 @@ def run_ours(args, rank, local_rank, world):
         for _ in range(args.e2e_steps):
             st_host = cg.replay_host(*hbuf, w.cap, POLICIES, trace_id_base=base,
                                      rand_seed=w.rand_seed, ovh=w.ovh, chunk=chunk,
-                                     summary=hsum, workspace=ws, stream=stream)
+                                     summary=hsum, workspace=ws, stream=stream,
+                                     kernel=args.kernel)
         e1.record(stream)
         torch.cuda.synchronize()
         e2e_ms = cgd.max_over_ranks(e0.elapsed_time(e1), dev)

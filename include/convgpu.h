@@ -95,8 +95,16 @@ typedef struct {
   uint64_t trace_id_base;    /* global id of trace 0 (sharding; Random-Fit counter) */
   uint64_t rand_seed;        /* Random-Fit Philox key (R6) */
   uint32_t ctx_overhead_mib; /* charged at a container's first ALLOC (66) */
-  uint32_t reserved0;        /* must be 0 */
+  uint32_t kernel_variant;   /* CONVGPU_KERNEL_*: 0 = auto (recommended) */
 } convgpu_traces_t;
+
+/* Replay kernel variants.  Results are bit-identical; only
+ * speed differs.  AUTO picks lane-per-trace when the batch fills the GPU. */
+enum {
+  CONVGPU_KERNEL_AUTO = 0,
+  CONVGPU_KERNEL_WARP_PER_TRACE = 1, /* one warp per trace, TMA-staged trace */
+  CONVGPU_KERNEL_LANE_PER_TRACE = 2  /* one lane per trace, 32 traces per warp */
+};
 
 /* Per-trace summary, 40 bytes. */
 typedef struct {
@@ -140,7 +148,7 @@ typedef struct {
  * policy: convgpu_policy_t.  n may be 0 (no-op).
  * Errors: -EINVAL for NULL traces/out/arrays, n_containers or n_ops out of
  * range, policy out of range, capacity out of range, overhead out of range,
- * reserved0 != 0, host pointers, range_digest without range_size; -ENODEV;
+ * kernel_variant > 2, host pointers, range_digest without range_size; -ENODEV;
  * -EIO (launch failure).
  */
 int convgpu_replay(const convgpu_traces_t *traces, uint64_t n, uint32_t capacity_mib,

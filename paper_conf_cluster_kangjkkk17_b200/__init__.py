@@ -26,6 +26,7 @@ FIFO, BEST_FIT, RECENT_FIT, RANDOM_FIT = 0, 1, 2, 3
 POLICY = {"fifo": FIFO, "best_fit": BEST_FIT, "recent_fit": RECENT_FIT, "random_fit": RANDOM_FIT}
 ALLOC, FREE, FINISH, NOP = 0, 1, 2, 3
 NONE32, NONE8 = 0xFFFFFFFF, 0xFF
+KERNEL = {"auto": 0, "warp": 1, "lane": 2}
 FLAG_NAMES = ("deadlock", "overcommit", "invalid_limit", "invalid_free", "unsorted_arrival",
               "tick_range", "bad_program")
 
@@ -48,7 +49,7 @@ class TracesT(C.Structure):
     _fields_ = [("arrival", C.c_void_p), ("limit", C.c_void_p), ("op_delta", C.c_void_p),
                 ("op_arg", C.c_void_p), ("n_containers", C.c_uint32), ("n_ops", C.c_uint32),
                 ("trace_id_base", C.c_uint64), ("rand_seed", C.c_uint64),
-                ("ctx_overhead_mib", C.c_uint32), ("reserved0", C.c_uint32)]
+                ("ctx_overhead_mib", C.c_uint32), ("kernel_variant", C.c_uint32)]
 
 
 class OutT(C.Structure):
@@ -144,13 +145,13 @@ class Traces:
     def nbytes(self) -> int:
         return sum(t.numel() * 4 for t in (self.arrival, self.limit, self.op_delta, self.op_arg))
 
-    def struct(self, rand_seed=0, ovh=0) -> TracesT:
+    def struct(self, rand_seed=0, ovh=0, kernel="auto") -> TracesT:
         for t in (self.arrival, self.limit, self.op_delta, self.op_arg):
             if not t.is_contiguous():
                 raise ConvgpuError("trace arrays must be contiguous")
         return TracesT(self.arrival.data_ptr(), self.limit.data_ptr(), self.op_delta.data_ptr(),
                        self.op_arg.data_ptr(), self.n, self.K, self.trace_id_base, rand_seed,
-                       ovh, 0)
+                       ovh, KERNEL[kernel])
 
 
 def empty_traces(count: int, n: int, K: int, device="cuda", trace_id_base=0) -> Traces:
@@ -235,10 +236,11 @@ def alloc_out(count: int, n: int, device="cuda", full=True, summary=True, stats=
 
 
 def replay(traces: Traces, capacity: int, policy, out: ReplayOut, rand_seed: int = 0,
-           ovh: int = 0, stream=None) -> ReplayOut:
+           ovh: int = 0, stream=None, kernel: str = "auto") -> ReplayOut:
     """Replay every trace of `traces` under `policy` (convgpu_replay).  Outputs
-    go to the tensors of `out`; out.stats is accumulated (zero it first)."""
-    tr = traces.struct(rand_seed, ovh)
+    go to the tensors of `out`; out.stats is accumulated (zero it first).
+    kernel: "auto" | "warp" (warp per trace) | "lane" (lane per trace)."""
+    tr = traces.struct(rand_seed, ovh, kernel)
     o = OutT(_ptr(out.admit_tick), _ptr(out.admit_rank), _ptr(out.wait), _ptr(out.finish),
              _ptr(out.summary), _ptr(out.stats), _ptr(out.range_digest), out.range_size,
              _stream_handle(stream))
@@ -249,7 +251,8 @@ def replay(traces: Traces, capacity: int, policy, out: ReplayOut, rand_seed: int
 
 def replay_host(arrival, limit, delta, arg, capacity: int, policies=("fifo",), *,
                 trace_id_base=0, rand_seed=0, ovh=0, chunk: int = 1 << 17,
-                summary: Optional[np.ndarray] = None, workspace=None, stream=None):
+                summary: Optional[np.ndarray] = None, workspace=None, stream=None,
+                kernel: str = "auto"):
     """End-to-end replay from HOST arrays (numpy or pinned torch; uint32/int32
     in the layouts of include/convgpu.h) through convgpu_replay_host: chunks
     are copied in, replayed under every policy in `policies` while resident,
@@ -275,7 +278,7 @@ def replay_host(arrival, limit, delta, arg, capacity: int, policies=("fifo",), *
         mask |= 1 << _pol(q)
     npol = bin(mask).count("1")
     tr = TracesT(ptr(arrs[0]), ptr(arrs[1]), ptr(arrs[2]), ptr(arrs[3]), n, K, trace_id_base,
-                 rand_seed, ovh, 0)
+                 rand_seed, ovh, KERNEL[kernel])
     need = host_workspace_bytes(n, K, chunk, npol)
     if workspace is None or workspace.numel() < need:
         workspace = torch.empty(need, dtype=torch.uint8, device="cuda")

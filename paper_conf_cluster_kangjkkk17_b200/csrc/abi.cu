@@ -54,7 +54,7 @@ int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
   if (policy < 0 || policy > 3) return -EINVAL;
   if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
   if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
-  if (t->reserved0 != 0) return -EINVAL;
+  if (t->kernel_variant > CONVGPU_KERNEL_LANE_PER_TRACE) return -EINVAL;
   return 0;
 }
 
@@ -76,6 +76,25 @@ convgpu::ReplayArgs make_args(const convgpu_traces_t* t, uint64_t n, uint32_t ca
 bool use_bulk(const convgpu::ReplayArgs& a) {
   return (a.n % 4u) == 0 && aligned16(a.arrival) && aligned16(a.limit) && aligned16(a.delta) &&
          aligned16(a.arg);
+}
+
+// Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, profiles/):
+// lane-per-trace needs enough traces to give every SM several CTAs; it wins
+// for the O(1)-selection policies (FIFO, Random-Fit).  Best-Fit and
+// Recent-Fit scan the paused set per selection, which diverges across lanes,
+// so they stay on warp-per-trace.
+uint32_t auto_variant(uint64_t count, int policy) {
+  int dev = 0, sms = 148;
+  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const bool big = count >= (uint64_t)sms * 2 * convgpu::kLptThreads * 4;
+  const bool o1 = policy == CONVGPU_FIFO || policy == CONVGPU_RANDOM_FIT;
+  return (big && o1) ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
+}
+
+cudaError_t launch_any(const convgpu::ReplayArgs& a, int policy, uint32_t variant, cudaStream_t s) {
+  if (variant == CONVGPU_KERNEL_AUTO) variant = auto_variant(a.count, policy);
+  if (variant == CONVGPU_KERNEL_LANE_PER_TRACE) return convgpu::launch_replay_lpt(a, policy, s);
+  return convgpu::launch_replay(a, policy, use_bulk(a), s);
 }
 
 }  // namespace
@@ -118,7 +137,7 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   a.wait = out->wait; a.finish = out->finish;
   a.summary = out->summary; a.stats = out->stats;
   a.range_digest = out->range_digest; a.range_size = out->range_size;
-  cudaError_t e = convgpu::launch_replay(a, policy, use_bulk(a), (cudaStream_t)out->stream);
+  cudaError_t e = launch_any(a, policy, traces->kernel_variant, (cudaStream_t)out->stream);
   return e == cudaSuccess ? 0 : fail_cuda(e, "replay launch");
 }
 
@@ -227,7 +246,7 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
-      e = convgpu::launch_replay(a, pols[q], use_bulk(a), cs);
+      e = launch_any(a, pols[q], ht->kernel_variant, cs);
     }
     if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
     if (e == cudaSuccess && host_summary) {

@@ -8,7 +8,8 @@
 
 namespace convgpu {
 
-constexpr int kReplayThreads = 128;  // 4 warps, one trace each at a time
+constexpr int kReplayThreads = 128;  // warp-per-trace: 4 warps, one trace each at a time
+constexpr int kLptThreads = 64;      // lane-per-trace: 2 warps, 64 traces at a time
 
 struct ReplayArgs {
   const uint32_t *arrival, *limit, *delta, *arg;
@@ -27,6 +28,7 @@ struct ReplayArgs {
 };
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream);
+cudaError_t launch_replay_lpt(const ReplayArgs& a, int policy, cudaStream_t stream);
 
 struct GenArgs {
   convgpu_gen_params_t p;

@@ -63,7 +63,7 @@ def _traces(**kw):
 
 @pytest.mark.parametrize("kw", [dict(n_containers=0), dict(n_containers=65), dict(n_ops=0),
                                 dict(n_ops=9), dict(arrival=None), dict(op_arg=None),
-                                dict(reserved0=1), dict(ctx_overhead_mib=1 << 30)])
+                                dict(kernel_variant=3), dict(ctx_overhead_mib=1 << 30)])
 def test_replay_rejects_bad_shape_before_touching_the_device(so, kw):
     out = cg.OutT()
     assert so.convgpu_replay(C.byref(_traces(**kw)), 10, 1000, 0, C.byref(out)) == -errno.EINVAL

@@ -22,11 +22,15 @@ def cg():
     return m
 
 
-def _gpu_replay(cg, tr, cap, policy, seed=0, ovh=0, full=True, range_size=0, range_count=0):
+KERNELS = ["warp", "lane"]
+
+
+def _gpu_replay(cg, tr, cap, policy, seed=0, ovh=0, full=True, range_size=0, range_count=0,
+                kernel="auto"):
     import torch
     out = cg.alloc_out(tr.count, tr.n, full=full, range_count=range_count,
                        range_size=range_size)
-    cg.replay(tr, cap, policy, out, rand_seed=seed, ovh=ovh)
+    cg.replay(tr, cap, policy, out, rand_seed=seed, ovh=ovh, kernel=kernel)
     torch.cuda.synchronize()
     return out
 
@@ -76,12 +80,13 @@ def test_generator_jitter_and_64bit_ids(cg, orc):
 
 # ---------------------------------------------------------------- replay
 @pytest.mark.parametrize("policy", POLS)
-def test_fig3_on_gpu(cg, orc, policy):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_fig3_on_gpu(cg, orc, kernel, policy):
     from conftest import golden
     f = W.fig3_fixture()
     tr = cg.traces_from_numpy(f["arrival"][None], f["limit"][None], f["delta"][None],
                               f["arg"][None])
-    out = _gpu_replay(cg, tr, f["cap"], policy)
+    out = _gpu_replay(cg, tr, f["cap"], policy, kernel=kernel)
     g = golden("fig3.json")["expected_all_policies"]
     s = out.summary_np()[0]
     full = out.full_np()
@@ -112,61 +117,66 @@ EDGE = [  # (n, K, cap, ovh, mode, count)
 
 @pytest.mark.parametrize("case", EDGE, ids=lambda c: f"n{c[0]}K{c[1]}{c[4]}")
 @pytest.mark.parametrize("policy", POLS)
-def test_edge_batches(cg, orc, case, policy):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_edge_batches(cg, orc, kernel, case, policy):
     n, K, cap, ovh, mode, count = case
     b = W.random_batch(1000 + n * 10 + K, count, n, K, cap, ovh=ovh, mode=mode,
                        limit_choices=range(0, cap + 1))
     base = 5_000_000_000 + n
     ref = orc.replay_batch(b, cap, policy, tid_base=base, rand_seed=99 + n, ovh=ovh)
     tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=base)
-    out = _gpu_replay(cg, tr, cap, policy, seed=99 + n, ovh=ovh)
+    out = _gpu_replay(cg, tr, cap, policy, seed=99 + n, ovh=ovh, kernel=kernel)
     _compare(cg, out, ref)
     _compare_stats(cg, out, ref["stats"])
 
 
 @pytest.mark.parametrize("policy", POLS)
-def test_config1_full(cg, orc, policy):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_config1_full(cg, orc, kernel, policy):
     """BASELINE config [1]: 10^4 traces x 16 containers, every output field."""
     w = W.CONFIGS["c1"]
     N = w.n_traces
     ref = orc.replay_range(w, policy, 0, N, full=True)
     tr = cg.generate(w.gen, 0, N)
-    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel=kernel)
     _compare(cg, out, ref)
     _compare_stats(cg, out, ref["stats"])
     assert ref["stats"]["flag_count"][0] == 0  # no deadlock (P:7)
 
 
 @pytest.mark.parametrize("policy", POLS)
-def test_config2_window_with_ragged_tail(cg, orc, policy):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_config2_window_with_ragged_tail(cg, orc, kernel, policy):
     """Config [2] generator; a window of trace ids whose count is not a
     multiple of the warps in flight, at an unaligned 64-bit base."""
     w = W.CONFIGS["c2"]
     base, N = 987_654_321_001, 4_741
     ref = orc.replay_range(w, policy, base, base + N, full=True)
     tr = cg.generate(w.gen, base, N)
-    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel=kernel)
     _compare(cg, out, ref)
     _compare_stats(cg, out, ref["stats"])
 
 
 @pytest.mark.parametrize("policy", POLS)
-def test_mimic_with_overhead(cg, orc, policy):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_mimic_with_overhead(cg, orc, kernel, policy):
     w = W.CONFIGS["mimic"]
     N = 3000
     ref = orc.replay_range(w, policy, 0, N, full=True)
     tr = cg.generate(w.gen, 0, N)
-    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, ovh=w.ovh)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, ovh=w.ovh, kernel=kernel)
     _compare(cg, out, ref)
 
 
 @pytest.mark.parametrize("policy", POLS)
 @pytest.mark.parametrize("rho", [1, 4, 8])
-def test_rho_sweep_window(cg, orc, policy, rho):
+@pytest.mark.parametrize("kernel", KERNELS)
+def test_rho_sweep_window(cg, orc, kernel, policy, rho):
     w = W.rho_sweep(rho, rand_seed=rho * 7 + 1)
     ref = orc.replay_range(w, policy, 10_000, 11_500, full=True)
     tr = cg.generate(w.gen, 10_000, 1_500)
-    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel=kernel)
     _compare(cg, out, ref)
 
 
