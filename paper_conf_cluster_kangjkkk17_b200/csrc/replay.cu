@@ -1,23 +1,26 @@
 // replay.cu — the hot path: batched replay of ConVGPU's GPU-memory scheduler
-// (§III-D, Fig. 3) on sm_100a.
+// (§III-D, Fig. 3) on sm_100a, one warp per
+// trace.
 //
-// Design (DESIGN.md §Kernels):
-//  * one warp per trace, persistent grid-stride over traces;
+// Design (DESIGN.md §6):
+//  * persistent grid-stride loop over traces, one trace per warp at a time;
 //  * the next trace's SoA arrays are prefetched into a per-warp shared-memory
 //    double buffer by the bulk-copy (TMA) engine — cp.async.bulk completing
 //    on an mbarrier — while the warp replays the current trace;
 //  * event keys (tick << 6 | container) live in registers, two containers
-//    per lane; the next event is one __reduce_min_sync (redux.sync.min);
-//  * per-container ledger (used, wait, admission, op cursor, flags) lives in
-//    shared memory and is updated by warp-uniform code (broadcast reads), the
-//    scheduler ledger (free memory, fill target, counters) in uniform
-//    registers — no divergence in the event loop;
+//    per lane; the next event is one redux.sync.min;
+//  * each container's hot state is one 16-byte record {state, current op
+//    word, delta to its next op, limit} in shared memory: an event is one
+//    broadcast LDS.128, an advance one STS.128 (the next op's word/delta come
+//    from the staged trace); the scheduler ledger (free memory, fill target,
+//    counters, the 64-bit paused mask) is warp-uniform in registers, so the
+//    event loop never diverges;
 //  * policy selection is lane-parallel: FIFO = find-first-set of
 //    the paused mask, Best-Fit = two packed redux (max fitting shortfall,
 //    else min shortfall), Recent-Fit = redux.max over packed suspension
-//    numbers, Random-Fit = Philox draw + popc + fns over the paused mask;
-//  * outputs, the R20 digest, and a warp -> block -> grid statistics
-//    reduction are fused into the trace epilogue / kernel tail.
+//    numbers, Random-Fit = Philox draw + popc + fns;
+//  * outputs, the R20 digest and a warp -> block -> grid statistics reduction
+//    are fused into the trace epilogue / kernel tail.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -25,15 +28,17 @@
 #include "internal.h"
 
 namespace convgpu {
+namespace wpt {
 
-// Per-container state word in shared memory.
-enum : uint32_t {
-  kStK = 0xFu,              // index of the next op
-  kStArrived = 1u << 4,
-  kStFirst = 1u << 5,       // first allocation of the pid done
-  kStAdmitted = 1u << 6,    // assignment == declared limit
-  kStPaused = 1u << 7,      // allocation reply withheld
-};
+// state word: used (26 bits) | k << 26 (3 bits) | FIRST | PAUSED | ADMITTED;
+// PAUSED|ADMITTED together (impossible for a live container) = not arrived.
+constexpr uint32_t kUsedMask = (1u << 26) - 1;
+constexpr uint32_t kKShift = 26;
+constexpr uint32_t kKMask = 7u << kKShift;
+constexpr uint32_t kFirst = 1u << 29;
+constexpr uint32_t kPaused = 1u << 30;
+constexpr uint32_t kAdmitted = 1u << 31;
+constexpr uint32_t kNotArrived = kPaused | kAdmitted;
 constexpr uint32_t kTargetNone = 64u;
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
@@ -45,12 +50,18 @@ struct WarpStats {  // 96 B, per warp, shared memory
 };
 static_assert(sizeof(WarpStats) == 96, "WarpStats layout");
 
-constexpr uint32_t kHeaderBytes = 128;         // 2 mbarriers + WarpStats + range acc
-constexpr uint32_t kStateWords = 6 * 64;       // used, wait, admit, st, fin, seq
+// Per-warp shared memory: header (2 mbarriers, WarpStats, range accumulator)
+// | cs[64] {state, cw, nd, L} | cx[64] {wait, adm} | 2 x staged trace.
+// cs.nd: delta to add at the container's next scheduling (d_0 before
+//        arrival, then d_{k+1}); after FINISH it holds the finish tick.
+// cx.wait: d_1 before arrival, then the suspended-time accumulator.
+// cx.adm: admission (tick << 6 | rank); suspension number while paused.
+constexpr uint32_t kHeaderBytes = 128;
+constexpr uint32_t kCsBytes = 64 * 16, kCxBytes = 64 * 8;
 
 __host__ __device__ inline uint32_t in_words(uint32_t n, uint32_t K) { return (2 + 2 * K) * n; }
 __host__ __device__ inline uint32_t warp_region_bytes(uint32_t n, uint32_t K) {
-  uint32_t b = kHeaderBytes + kStateWords * 4 + 2 * in_words(n, K) * 4;
+  uint32_t b = kHeaderBytes + kCsBytes + kCxBytes + 2 * in_words(n, K) * 4;
   return (b + 15u) & ~15u;
 }
 
@@ -83,26 +94,34 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+__device__ __forceinline__ uint32_t redux_min(uint32_t v) {
+  uint32_t r;
+  asm volatile("redux.sync.min.u32 %0, %1, 0xffffffff;" : "=r"(r) : "r"(v));
+  return r;
+}
+__device__ __forceinline__ uint32_t redux_max(uint32_t v) {
+  uint32_t r;
+  asm volatile("redux.sync.max.u32 %0, %1, 0xffffffff;" : "=r"(r) : "r"(v));
+  return r;
+}
 
 // ---------------------------------------------------------------- kernel
-template <int POLICY, bool BULK>
+// NF: compile-time container count (64) or 0 = runtime p.n.
+template <int POLICY, bool BULK, int NF>
 __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const uint32_t lane = threadIdx.x & 31u;
+  const uint32_t lane = threadIdx.x & 31u, lane32 = lane + 32u;
   const uint32_t wib = threadIdx.x >> 5;
-  const uint32_t n = p.n, K = p.K;
+  const uint32_t n = NF ? (uint32_t)NF : p.n;
+  const uint32_t K = p.K, cap = p.cap, ovh = p.ovh;
   const uint32_t IN = in_words(n, K);
   unsigned char* base = smem + wib * warp_region_bytes(n, K);
   uint64_t* mbar = reinterpret_cast<uint64_t*>(base);
   WarpStats* ws = reinterpret_cast<WarpStats*>(base + 16);
   unsigned long long* racc = reinterpret_cast<unsigned long long*>(base + 112);  // [cur, acc]
-  uint32_t* s_used = reinterpret_cast<uint32_t*>(base + kHeaderBytes);
-  uint32_t* s_wait = s_used + 64;
-  uint32_t* s_admit = s_used + 128;  // tick << 6 | rank, or kKeyNone
-  uint32_t* s_st = s_used + 192;
-  uint32_t* s_fin = s_used + 256;
-  uint32_t* s_seq = s_used + 320;
-  uint32_t* inbuf = s_used + kStateWords;  // [2][IN]
+  uint4* cs = reinterpret_cast<uint4*>(base + kHeaderBytes);
+  uint2* cx = reinterpret_cast<uint2*>(base + kHeaderBytes + kCsBytes);
+  uint32_t* inbuf = reinterpret_cast<uint32_t*>(base + kHeaderBytes + kCsBytes + kCxBytes);
 
   const uint64_t warps_per_block = blockDim.x >> 5;
   const uint64_t gw = (uint64_t)blockIdx.x * warps_per_block + wib;
@@ -168,16 +187,15 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
     const uint32_t* R = A + 2 * n + K * n;
     const uint64_t tid = p.tid_base + i;
 
-    // ---- per-trace init + static validation ----
+    // ---- per-trace init + static validation (DESIGN.md §2 Flags) ----
     uint32_t key0 = kKeyNone, key1 = kKeyNone;
     uint32_t bad = 0, lsum = 0, lmax = 0;
 #pragma unroll
     for (uint32_t s = 0; s < 2; ++s) {
       const uint32_t c = lane + 32u * s;
-      s_used[c] = 0; s_wait[c] = 0; s_admit[c] = kKeyNone; s_st[c] = 0; s_fin[c] = 0; s_seq[c] = 0;
       if (c < n) {
-        const uint32_t a = A[c];
-        if (Lm[c] > p.cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+        const uint32_t a = A[c], L = Lm[c];
+        if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
         if (c > 0 && a < A[c - 1]) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
         lmax = max(lmax, a);
         for (uint32_t k = 0; k < K; ++k) {
@@ -185,6 +203,8 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
           const bool fin = (R[k * n + c] >> 30) == CONVGPU_OP_FINISH;
           if (fin != (k + 1 == K)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
         }
+        cs[c] = make_uint4(kNotArrived, R[c], D[c], L);
+        cx[c] = make_uint2(K > 1 ? D[n + c] : 0u, kKeyNone);
         const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
         if (s == 0) key0 = key; else key1 = key;
       }
@@ -198,118 +218,131 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
     __syncwarp();
 
     // ---- uniform scheduler ledger (D4, D1 target, counters) ----
-    uint32_t free_mem = p.cap, target = kTargetNone, a_tg = 0, used_total = 0;
+    uint32_t free_mem = cap, target = kTargetNone, a_tg = 0, used_total = 0;
     uint32_t seq = 0, rank = 0, draws = 0, n_rej = 0, n_sel = 0;
     uint32_t peak_res = 0, peak_used = 0, live = n, events = 0;
     uint32_t pm_lo = 0, pm_hi = 0;  // paused set (D3) as a 64-bit mask
 
-    auto set_key = [&](uint32_t c, uint32_t k) {
-      if (lane == (c & 31u)) {
-        if (c & 32u) key1 = k; else key0 = k;
-      }
-    };
-
     if (flags == 0) {
       for (;;) {
-        const uint32_t kmin = __reduce_min_sync(kFull, min(key0, key1));
+        const uint32_t kmin = redux_min(min(key0, key1));
         if (kmin == kKeyNone) {
           if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
           break;
         }
         const uint32_t t = kmin >> 6, c = kmin & 63u;
         ++events;
-        uint32_t st = s_st[c];
-        const uint32_t L = Lm[c];
+        const uint4 s = cs[c];
+        uint32_t ust = s.x;
+        const uint32_t L = s.w;
         uint32_t nk = kKeyNone;
         bool disp = false;
-        if (!(st & kStArrived)) {
+        if ((ust & kNotArrived) == kNotArrived) {
           // ARRIVE (Fig. 3b/3c; R2)
           const uint32_t g = (target == kTargetNone) ? min(L, free_mem) : 0u;
           free_mem -= g;
-          st |= kStArrived;
+          peak_res = max(peak_res, cap - free_mem);
+          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+          uint32_t adm = kKeyNone;
+          ust = 0;
           if (g == L) {
-            s_admit[c] = (t << 6) | rank; ++rank; st |= kStAdmitted;
+            adm = (t << 6) | rank; ++rank; ust = kAdmitted;
           } else if (g > 0) {
             target = c; a_tg = g;
           }
-          nk = ((t + D[c]) << 6) | c;
+          const uint32_t d1 = cx[c].x;
+          cx[c] = make_uint2(0u, adm);
+          cs[c] = make_uint4(ust, s.y, d1, L);
+          nk = ((t + s.z) << 6) | c;
         } else {
-          uint32_t k = st & kStK;
-          const uint32_t w = R[k * n + c];
-          const uint32_t kind = w >> 30, r = w & kSizeMask;
+          const uint32_t cw = s.y;
+          const uint32_t kind = cw >> 30, r = cw & kSizeMask, used = ust & kUsedMask;
           bool adv = true;
           if (kind == CONVGPU_OP_ALLOC) {
-            const uint32_t used = s_used[c];
-            const uint32_t need = used + r + ((st & kStFirst) ? 0u : p.ovh);
-            const uint32_t a = (st & kStAdmitted) ? L : (c == target ? a_tg : 0u);
+            const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
+            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
             if (need > L) {
               ++n_rej;  // R10
             } else if (need <= a) {
-              s_used[c] = need; used_total += need - used; st |= kStFirst;
+              used_total += need - used;
+              peak_used = max(peak_used, used_total);
+              if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+              ust = (ust & ~kUsedMask) | need | kFirst;
             } else {  // pause: reply withheld
-              st |= kStPaused;
-              s_wait[c] -= t;
-              if (POLICY == CONVGPU_RECENT_FIT) s_seq[c] = seq;
+              ust |= kPaused;
+              const uint32_t wv = cx[c].x - t;
+              cx[c] = make_uint2(wv, POLICY == CONVGPU_RECENT_FIT ? seq : kKeyNone);
               ++seq;
               if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
               adv = false;
               disp = (target == kTargetNone);
+              cs[c].x = ust;
             }
           } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
-            const uint32_t used = s_used[c];
             if (r > used) { flags |= CONVGPU_FLAG_INVALID_FREE; break; }
-            s_used[c] = used - r; used_total -= r;
+            ust -= r;
+            used_total -= r;
           } else if (kind == CONVGPU_OP_FINISH) {  // P:110, R18
-            const uint32_t a = (st & kStAdmitted) ? L : (c == target ? a_tg : 0u);
+            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
             free_mem += a;
-            used_total -= s_used[c];
-            s_used[c] = 0;
-            s_fin[c] = t;
+            used_total -= used;
             --live;
             if (c == target) { target = kTargetNone; a_tg = 0; }  // R20
+            cs[c] = make_uint4(ust & ~kUsedMask, cw, t, L);  // nd := finish tick
             adv = false;
             disp = true;
           }
           if (adv) {
-            ++k;
-            st = (st & ~kStK) | k;
-            nk = ((t + D[k * n + c]) << 6) | c;
+            const uint32_t k = ((ust >> kKShift) & 7u) + 1u;
+            nk = ((t + s.z) << 6) | c;
+            ust = (ust & ~kKMask) | (k << kKShift);
+            const uint32_t ncw = R[k * n + c];
+            const uint32_t nnd = (k + 1 < K) ? D[(k + 1) * n + c] : 0u;
+            cs[c] = make_uint4(ust, ncw, nnd, L);
           }
         }
-        s_st[c] = st;
-        set_key(c, nk);
+        key0 = (c == lane) ? nk : key0;
+        key1 = (c == lane32) ? nk : key1;
 
         // ---- DISPATCH (Fig. 3d; R1, R9) ----
         if (disp) {
           for (;;) {
             if (target != kTargetNone) {
-              const uint32_t tg = target, Lt = Lm[tg];
+              const uint32_t tg = target;
+              uint4 st = cs[tg];
+              const uint32_t Lt = st.w;
               const uint32_t g = min(free_mem, Lt - a_tg);
               a_tg += g;
               free_mem -= g;
-              uint32_t stt = s_st[tg];
-              if (stt & kStPaused) {
-                uint32_t kt = stt & kStK;
-                const uint32_t pend = (R[kt * n + tg] & kSizeMask) + ((stt & kStFirst) ? 0u : p.ovh);
-                const uint32_t ut = s_used[tg];
-                if (ut + pend <= a_tg) {  // RESUME (R9)
-                  s_used[tg] = ut + pend;
+              peak_res = max(peak_res, cap - free_mem);
+              if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+              uint32_t ut = st.x;
+              if (ut & kPaused) {
+                const uint32_t pend = (st.y & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
+                const uint32_t uu = ut & kUsedMask;
+                if (uu + pend <= a_tg) {  // RESUME (R9)
                   used_total += pend;
-                  s_wait[tg] += t;
+                  peak_used = max(peak_used, used_total);
+                  if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+                  cx[tg] = make_uint2(cx[tg].x + t, kKeyNone);
                   if (tg < 32) pm_lo &= ~(1u << tg); else pm_hi &= ~(1u << (tg - 32));
-                  ++kt;
-                  stt = (stt & ~(kStK | kStPaused)) | kStFirst | kt;
-                  set_key(tg, ((t + D[kt * n + tg]) << 6) | tg);
+                  const uint32_t k = ((ut >> kKShift) & 7u) + 1u;
+                  ut = (ut & ~(kUsedMask | kKMask | kPaused)) | (uu + pend) | kFirst | (k << kKShift);
+                  const uint32_t nkt = ((t + st.z) << 6) | tg;
+                  key0 = (tg == lane) ? nkt : key0;
+                  key1 = (tg == lane32) ? nkt : key1;
+                  st.y = R[k * n + tg];
+                  st.z = (k + 1 < K) ? D[(k + 1) * n + tg] : 0u;
                 }
               }
               if (a_tg == Lt) {  // fully guaranteed: admit, cascade leftover
-                s_admit[tg] = (t << 6) | rank; ++rank;
-                s_st[tg] = stt | kStAdmitted;
+                cx[tg].y = (t << 6) | rank; ++rank;
+                cs[tg] = make_uint4(ut | kAdmitted, st.y, st.z, Lt);
                 target = kTargetNone;
                 a_tg = 0;
                 continue;
               }
-              s_st[tg] = stt;
+              cs[tg] = make_uint4(ut, st.y, st.z, Lt);
               break;
             }
             if ((pm_lo | pm_hi) == 0u) break;
@@ -317,29 +350,25 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             uint32_t sel;
             if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
               sel = pm_lo ? (uint32_t)(__ffs(pm_lo) - 1) : 32u + (uint32_t)(__ffs(pm_hi) - 1);
-            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4
+            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
               uint32_t vf = 0, vm = kKeyNone;
-#pragma unroll
-              for (uint32_t s = 0; s < 2; ++s) {
-                const uint32_t c2 = lane + 32u * s;
-                const uint32_t m = s ? pm_hi : pm_lo;
-                if ((m >> lane) & 1u) {
-                  const uint32_t need = Lm[c2];  // shortfall L - a, a = 0 when selectable
-                  if (need <= free_mem) vf = max(vf, (need << 6) | (63u - c2));
-                  vm = min(vm, (need << 6) | c2);
-                }
+              if ((pm_lo >> lane) & 1u) {
+                const uint32_t need = Lm[lane];
+                if (need <= free_mem) vf = (need << 6) | (63u - lane);
+                vm = (need << 6) | lane;
               }
-              const uint32_t kf = __reduce_max_sync(kFull, vf);
-              if (kf) {
-                sel = 63u - (kf & 63u);
-              } else {
-                sel = __reduce_min_sync(kFull, vm) & 63u;
+              if (lane32 < n && ((pm_hi >> lane) & 1u)) {
+                const uint32_t need = Lm[lane32];
+                if (need <= free_mem) vf = max(vf, (need << 6) | (63u - lane32));
+                vm = min(vm, (need << 6) | lane32);
               }
+              const uint32_t kf = redux_max(vf);
+              sel = kf ? 63u - (kf & 63u) : (redux_min(vm) & 63u);
             } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
               uint32_t v = 0;
-              if ((pm_lo >> lane) & 1u) v = ((s_seq[lane] + 1u) << 6) | lane;
-              if ((pm_hi >> lane) & 1u) v = max(v, ((s_seq[lane + 32] + 1u) << 6) | (lane + 32u));
-              sel = __reduce_max_sync(kFull, v) & 63u;
+              if ((pm_lo >> lane) & 1u) v = ((cx[lane].y + 1u) << 6) | lane;
+              if (lane32 < n && ((pm_hi >> lane) & 1u)) v = max(v, ((cx[lane32].y + 1u) << 6) | lane32);
+              sel = redux_max(v) & 63u;
             } else {  // RANDOM_FIT (R6)
               const uint32_t clo = __popc(pm_lo);
               const uint32_t m = clo + __popc(pm_hi);
@@ -354,14 +383,11 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             ++n_sel;
           }
         }
-        const uint32_t reserved = p.cap - free_mem;
-        peak_res = max(peak_res, reserved);
-        peak_used = max(peak_used, used_total);
-        if (free_mem > p.cap || used_total > reserved) flags |= CONVGPU_FLAG_OVERCOMMIT;
       }
     }
 
     // ---- epilogue: outputs, digest (R20), statistics ----
+    __syncwarp();
     const bool stopped = (flags & kStopMask) != 0;
     if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
     uint64_t dig = 0;
@@ -372,10 +398,11 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
       if (c < n) {
         uint32_t at = kKeyNone, ar = 0xFFu, wt = 0, fn = 0;
         if (!stopped) {
-          const uint32_t adm = s_admit[c];
-          if (adm != kKeyNone) { at = adm >> 6; ar = adm & 63u; }
-          wt = s_wait[c];
-          fn = s_fin[c];
+          const uint4 st = cs[c];
+          const uint2 sx = cx[c];
+          if (st.x & kAdmitted) { at = sx.y >> 6; ar = sx.y & 63u; }
+          wt = sx.x;
+          fn = st.z;
         }
         const uint64_t gi = i * n + c;
         if (p.admit_tick) p.admit_tick[gi] = at;
@@ -459,11 +486,11 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
 }
 
 // ---------------------------------------------------------------- launcher
-template <int POLICY, bool BULK>
+template <int POLICY, bool BULK, int NF>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
   const uint32_t warps = kReplayThreads / 32;
   const size_t smem = (size_t)warps * warp_region_bytes(a.n, a.K);
-  auto kern = replay_kernel<POLICY, BULK>;
+  auto kern = replay_kernel<POLICY, BULK, NF>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0, per_sm = 0;
@@ -482,16 +509,20 @@ static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
   return cudaGetLastError();
 }
 
+template <int POLICY>
+static cudaError_t launch_p(const ReplayArgs& a, bool bulk, cudaStream_t stream) {
+  if (a.n == 64) return bulk ? launch_t<POLICY, true, 64>(a, stream) : launch_t<POLICY, false, 64>(a, stream);
+  return bulk ? launch_t<POLICY, true, 0>(a, stream) : launch_t<POLICY, false, 0>(a, stream);
+}
+
+}  // namespace wpt
+
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream) {
-  switch (policy * 2 + (bulk ? 1 : 0)) {
-    case 0: return launch_t<CONVGPU_FIFO, false>(a, stream);
-    case 1: return launch_t<CONVGPU_FIFO, true>(a, stream);
-    case 2: return launch_t<CONVGPU_BEST_FIT, false>(a, stream);
-    case 3: return launch_t<CONVGPU_BEST_FIT, true>(a, stream);
-    case 4: return launch_t<CONVGPU_RECENT_FIT, false>(a, stream);
-    case 5: return launch_t<CONVGPU_RECENT_FIT, true>(a, stream);
-    case 6: return launch_t<CONVGPU_RANDOM_FIT, false>(a, stream);
-    case 7: return launch_t<CONVGPU_RANDOM_FIT, true>(a, stream);
+  switch (policy) {
+    case CONVGPU_FIFO: return wpt::launch_p<CONVGPU_FIFO>(a, bulk, stream);
+    case CONVGPU_BEST_FIT: return wpt::launch_p<CONVGPU_BEST_FIT>(a, bulk, stream);
+    case CONVGPU_RECENT_FIT: return wpt::launch_p<CONVGPU_RECENT_FIT>(a, bulk, stream);
+    case CONVGPU_RANDOM_FIT: return wpt::launch_p<CONVGPU_RANDOM_FIT>(a, bulk, stream);
   }
   return cudaErrorInvalidValue;
 }
