@@ -80,14 +80,13 @@ bool use_bulk(const convgpu::ReplayArgs& a) {
 
 // Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, profiles/):
 // lane-per-trace needs enough traces to give every SM several CTAs; it wins
-// for the O(1)-selection policies (FIFO, Random-Fit).  Best-Fit and
-// Recent-Fit scan the paused set per selection, which diverges across lanes,
-// so they stay on warp-per-trace.
+// for FIFO, Recent-Fit and Random-Fit.  Best-Fit's per-trace rank tables cost
+// occupancy and an O(n^2) init there, so it stays on warp-per-trace.
 uint32_t auto_variant(uint64_t count, int policy) {
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const bool big = count >= (uint64_t)sms * 2 * convgpu::kLptThreads * 4;
-  const bool o1 = policy == CONVGPU_FIFO || policy == CONVGPU_RANDOM_FIT;
+  const bool o1 = policy != CONVGPU_BEST_FIT;
   return (big && o1) ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
 }
 

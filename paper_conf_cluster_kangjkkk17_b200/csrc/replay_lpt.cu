@@ -1,24 +1,33 @@
 // replay_lpt.cu — lane-per-trace replay of ConVGPU's GPU-memory scheduler
 // (§III-D, Fig. 3) on sm_100a.
 //
-// The warp-per-trace kernel (replay.cu) spends ~85 warp instructions per
+// The warp-per-trace kernel (replay.cu) spends ~70 warp instructions per
 // event because one trace's event loop is inherently serial and all 32 lanes
-// execute it.  Here every LANE owns a trace, so each warp instruction
-// advances 32 independent traces:
+// execute it.  Here every LANE owns a trace, so one warp instruction advances
+// 32 independent traces:
 //  * per-container state lives in shared memory in a lane-interleaved layout
 //    (word w of container c of lane l at [(w*n + c)*32 + l]) — every access
 //    with an arbitrary per-lane container index is bank-conflict-free;
-//  * the next event is found with a two-level min: 8 group minima (8
-//    containers each) in registers, the 64 keys in shared memory; a key
-//    change re-mins one group (8 LDS + 7 IMNMX);
-//  * the op words of a container are fetched one op ahead with cp.async
-//    (global -> shared, no registers), one commit group per iteration; an
-//    event waits only for the group that can still be in flight for it;
-//  * outputs and the digest are produced in a per-trace epilogue, which all
-//    lanes run together (valid traces have exactly n*(1+K) events), and the
-//    statistics are reduced warp -> grid at the end.
+//  * the next event comes from a two-level min: 8 group minima (8 containers
+//    each) in registers, the keys in shared memory; a key change re-mins one
+//    group (8 LDS + 7 IMNMX);
+//  * each iteration is ONE micro-step per lane — an event, or one step of the
+//    DISPATCH loop that an event started — written branch-free (selects and
+//    predicated stores), so the 32 lanes stay converged whatever event kind
+//    each of them processes; one shared tail does the key update, group
+//    re-min and op prefetch;
+//  * a container's next op word / delta are fetched one op ahead with
+//    cp.async (global -> shared), one commit group per iteration; an event
+//    waits only when its container was prefetched in the previous iteration;
+//  * selection is O(1): FIFO = ffs of the paused mask, Random-Fit = Philox +
+//    popc + fns, Recent-Fit = a lazily-deleted suspension stack, Best-Fit =
+//    per-trace ranks of (limit, index) + a paused mask in rank order + a
+//    binary search of the free memory over the sorted limits;
+//  * suspended time is not tracked per event: wait = finish - arrival -
+//    sum(deltas) (R17) is recovered in the per-trace epilogue, which all
+//    lanes run together (they start and finish traces in lockstep).
 // Semantics are identical to replay.cu; parity is tested
-// against the oracle on both.
+// against the oracle for both kernels.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -32,21 +41,31 @@ namespace lpt {
 // PAUSED|ADMITTED together (impossible for a live container) = not arrived.
 constexpr uint32_t kUsedMask = (1u << 26) - 1;
 constexpr uint32_t kKShift = 26;
-constexpr uint32_t kKMask = 7u << kKShift;
+constexpr uint32_t kKOne = 1u << kKShift;
 constexpr uint32_t kFirst = 1u << 29;
 constexpr uint32_t kPaused = 1u << 30;
 constexpr uint32_t kAdmitted = 1u << 31;
 constexpr uint32_t kNotArrived = kPaused | kAdmitted;
-constexpr uint32_t kTargetNone = 64u;
+constexpr uint32_t kNoC = 64u;  // "no container" / no fill target
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
-constexpr int kWords = 7;  // key, L, ust, wait, adm, cw, nd
-enum { W_KEY = 0, W_L = 1, W_UST = 2, W_WAIT = 3, W_ADM = 4, W_CW = 5, W_ND = 6 };
-// Before arrival W_WAIT holds delta_0 and W_ADM delta_1 (K > 1).  While a
-// container is paused W_ADM holds its suspension number (Recent-Fit).  After
-// FINISH W_ND holds its finish tick.
+constexpr uint32_t kStack = 128;  // Recent-Fit suspension stack entries
 
-__host__ __device__ inline size_t warp_bytes(uint32_t n) { return (size_t)kWords * n * 32 * 4; }
+// shared-memory words per container
+enum { W_KEY = 0, W_L = 1, W_UST = 2, W_ADM = 3, W_CW = 4, W_ND = 5, W_BASE_WORDS = 6 };
+// W_ADM: d_1 before arrival; admission (tick << 6 | rank) once admitted;
+//        the suspension number while paused (Recent-Fit scan fallback).
+// W_ND:  delta to add at the container's next scheduling (d_0 before
+//        arrival, then d_{k+1}); the finish tick after FINISH.
+// Best-Fit adds W_RK (byte0 rank_of[j], byte1 gs[j], byte2 pi[j]) and W_LS
+// (limits sorted by (L, index)); Recent-Fit adds a kStack-byte stack.
+__host__ __device__ constexpr int extra_words(int policy) { return policy == CONVGPU_BEST_FIT ? 2 : 0; }
+
+__host__ __device__ inline size_t warp_bytes(int policy, uint32_t n) {
+  size_t b = (size_t)(W_BASE_WORDS + extra_words(policy)) * n * 32 * 4;
+  if (policy == CONVGPU_RECENT_FIT) b += kStack * 32;
+  return b;
+}
 
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -58,20 +77,44 @@ __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_grou
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
-template <int POLICY, int MODE>
+__device__ __forceinline__ bool bit64(uint32_t lo, uint32_t hi, uint32_t b) {
+  return ((b < 32 ? lo >> b : hi >> (b - 32)) & 1u) != 0;
+}
+__device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bool on) {
+  const uint32_t ml = (b < 32) ? (1u << b) : 0u, mh = (b >= 32 && b < 64) ? (1u << (b - 32)) : 0u;
+  lo = on ? (lo | ml) : (lo & ~ml);
+  hi = on ? (hi | mh) : (hi & ~mh);
+}
+__device__ __forceinline__ uint32_t ffs64(uint32_t lo, uint32_t hi) {  // lowest set bit, 64 if none
+  return lo ? (uint32_t)(__ffs(lo) - 1) : (hi ? 32u + (uint32_t)(__ffs(hi) - 1) : 64u);
+}
+__device__ __forceinline__ uint32_t fls64(uint32_t lo, uint32_t hi) {  // highest set bit
+  return hi ? 63u - (uint32_t)__clz(hi) : 31u - (uint32_t)__clz(lo);
+}
+__device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi) {  // bits < r
+  lo = r >= 32 ? 0xFFFFFFFFu : ((1u << r) - 1u);
+  hi = r >= 64 ? 0xFFFFFFFFu : (r <= 32 ? 0u : ((1u << (r - 32)) - 1u));
+}
+
+template <int POLICY>
 __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
   const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
   const uint32_t n = p.n, K = p.K, cap = p.cap, ovh = p.ovh;
-  uint32_t* const S = smem_w + (size_t)wib * kWords * n * 32 + lane;
+  uint32_t* const W0 = smem_w + (wib * warp_bytes(POLICY, n)) / 4;
+  uint32_t* const S = W0 + lane;
   uint32_t* const s_key = S + (size_t)W_KEY * n * 32;
   uint32_t* const s_L = S + (size_t)W_L * n * 32;
   uint32_t* const s_ust = S + (size_t)W_UST * n * 32;
-  uint32_t* const s_wait = S + (size_t)W_WAIT * n * 32;
   uint32_t* const s_adm = S + (size_t)W_ADM * n * 32;
   uint32_t* const s_cw = S + (size_t)W_CW * n * 32;
   uint32_t* const s_nd = S + (size_t)W_ND * n * 32;
+  uint32_t* const s_rk = S + (size_t)(W_BASE_WORDS + 0) * n * 32;  // Best-Fit only
+  uint32_t* const s_ls = S + (size_t)(W_BASE_WORDS + 1) * n * 32;  // Best-Fit only
+  uint8_t* const s_stk = reinterpret_cast<uint8_t*>(W0 + (size_t)W_BASE_WORDS * n * 32) + lane * 4;
 #define AT(arr, c) (arr)[(c) * 32u]
+#define RKB(j, b) reinterpret_cast<uint8_t*>(&AT(s_rk, (j)))[b]
+#define STK(e) s_stk[((e) >> 2) * 128u + ((e) & 3u)]
 
   const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
   uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -82,12 +125,12 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   uint32_t st_maxmk = 0, st_maxpk = 0;
   unsigned long long racc_r = ~0ull, racc = 0;
 
-  // per-trace scheduler ledger
+  // per-trace scheduler ledger (all in registers)
   uint32_t gmin[8];
-  uint32_t free_mem = 0, target = kTargetNone, a_tg = 0, used_total = 0, seq = 0, rank = 0,
-           draws = 0, n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0,
-           events = 0, a0 = 0;
-  uint32_t pm_lo = 0, pm_hi = 0, pfc_lo = 0, pfc_hi = 0;
+  uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, seq = 0, rank = 0, draws = 0,
+           n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
+  uint32_t pm_lo = 0, pm_hi = 0, pfc_lo = 0, pfc_hi = 0, pr_lo = 0, pr_hi = 0, sp = 0;
+  bool ru_scan = false;
   const uint32_t* trace_delta = nullptr;
   const uint32_t* trace_arg = nullptr;
 
@@ -100,16 +143,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
 #pragma unroll
     for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? m : gmin[j];
   };
-  auto prefetch = [&](uint32_t c, uint32_t k) {  // op k word, delta of op k+1
-    if (MODE == 2) {
-      if (k < K) AT(s_cw, c) = __ldg(trace_arg + (size_t)k * n + c);
-      if (k + 1 < K) AT(s_nd, c) = __ldg(trace_delta + (size_t)(k + 1) * n + c);
-      return;
-    }
-    if (k < K) cp_async4(&AT(s_cw, c), trace_arg + (size_t)k * n + c);
-    if (k + 1 < K) cp_async4(&AT(s_nd, c), trace_delta + (size_t)(k + 1) * n + c);
-    if (c < 32) pfc_lo |= 1u << c; else pfc_hi |= 1u << (c - 32);
-  };
+
   auto init = [&](uint64_t ti) {
     const uint32_t* A = p.arrival + ti * n;
     const uint32_t* Lg = p.limit + ti * n;
@@ -137,24 +171,44 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
       AT(s_key, c) = key;
       AT(s_L, c) = L;
       AT(s_ust, c) = kNotArrived;
-      AT(s_wait, c) = d0;
       AT(s_adm, c) = d1;
       AT(s_cw, c) = w0;
+      AT(s_nd, c) = d0;
       const uint32_t g = c >> 3;
 #pragma unroll
       for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? min(gmin[j], key) : gmin[j];
     }
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
+    if (POLICY == CONVGPU_BEST_FIT) {
+      // ranks of (L, index) ascending; gs = first rank with the same L
+      for (uint32_t c = 0; c < n; ++c) {
+        const uint32_t Lc = AT(s_L, c);
+        uint32_t lt = 0, eq = 0;
+        for (uint32_t d = 0; d < n; ++d) {
+          const uint32_t Ld = AT(s_L, d);
+          lt += (Ld < Lc) ? 1u : 0u;
+          eq += (Ld == Lc && d < c) ? 1u : 0u;
+        }
+        const uint32_t r = lt + eq;
+        RKB(c, 0) = (uint8_t)r;
+        RKB(r, 1) = (uint8_t)lt;
+        RKB(r, 2) = (uint8_t)c;
+        AT(s_ls, r) = Lc;
+      }
+    }
     flags = bad;
-    free_mem = cap; target = kTargetNone; a_tg = 0; used_total = 0; seq = 0; rank = 0;
-    draws = 0; n_rej = 0; n_sel = 0; peak_res = 0; peak_used = 0; live = n; events = 0;
-    a0 = __ldg(A);
-    pm_lo = pm_hi = pfc_lo = pfc_hi = 0;
+    free_mem = cap; target = kNoC; a_tg = 0; used_total = 0; seq = 0; rank = 0; draws = 0;
+    n_rej = 0; n_sel = 0; peak_res = 0; peak_used = 0; live = n; events = 0;
+    pm_lo = pm_hi = pfc_lo = pfc_hi = pr_lo = pr_hi = 0;
+    sp = 0;
+    ru_scan = false;
   };
+
   auto epilogue = [&](uint64_t ti) {
     cp_wait0();
     const bool stopped = (flags & kStopMask) != 0;
     if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
+    const uint32_t* A = p.arrival + ti * n;
     uint64_t dig = 0, swait = 0;
     uint32_t mfin = 0;
     const uint64_t ob = ti * n;
@@ -167,8 +221,10 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           at = adm >> 6;
           ar = adm & 63u;
         }
-        wt = AT(s_wait, c);
         fn = AT(s_nd, c);
+        uint32_t sd = __ldg(A + c);  // R17: wait = finish - arrival - sum of deltas
+        for (uint32_t k = 0; k < K; ++k) sd += __ldg(trace_delta + (size_t)k * n + c);
+        wt = fn - sd;
       }
       if (p.admit_tick) p.admit_tick[ob + c] = at;
       if (p.admit_rank) p.admit_rank[ob + c] = (uint8_t)ar;
@@ -179,7 +235,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
       mfin = max(mfin, fn);
       swait += wt;
     }
-    const uint32_t makespan = stopped ? 0u : mfin - a0;
+    const uint32_t makespan = stopped ? 0u : mfin - __ldg(A);
     dig += mix64(((uint64_t)makespan << 32) | peak_res);
     dig += mix64(((uint64_t)peak_used << 32) | flags);
     dig += mix64(swait);
@@ -209,199 +265,210 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     }
   };
 
-  bool have = i < p.count, halted = false;
-  if (have) { init(i); halted = flags != 0; }  // static flags stop before the first event
-  while (have) {
-    bool done = halted;
-    if (!done) {
-      // ---- next event: two-level min (a2) ----
-      const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
-      const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
-      const uint32_t kmin = min(min(m01, m23), min(m45, m67));
-      if (kmin == kKeyNone) {
-        if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
-        done = true;
-      } else {
-        const uint32_t t = kmin >> 6, c = kmin & 63u;
-        // the op data of c may still be in flight from the previous iteration
-        // groups older than the previous iteration's are complete after
-        // wait_group 1; the previous iteration's group (containers in pfc)
-        // may still be in flight
-        cp_wait1();
-        if (MODE == 1 || ((c < 32 ? (pfc_lo >> c) : (pfc_hi >> (c - 32))) & 1u)) cp_wait0();
-        pfc_lo = 0; pfc_hi = 0;
-        ++events;
-        uint32_t ust = AT(s_ust, c);
-        const uint32_t L = AT(s_L, c);
-        uint32_t nk = kKeyNone;
-        bool disp = false;
-        if ((ust & kNotArrived) == kNotArrived) {
-          // ARRIVE (P:98, P:149 Fig. 3b/3c; R2)
-          const uint32_t d0 = AT(s_wait, c), d1 = AT(s_adm, c);
-          const uint32_t g = (target == kTargetNone) ? min(L, free_mem) : 0u;
-          free_mem -= g;
-          uint32_t adm = kKeyNone;
-          ust = 0;
-          if (g == L) {
-            adm = (t << 6) | rank; ++rank; ust = kAdmitted;
-          } else if (g > 0) {
-            target = c; a_tg = g;
-          }
-          AT(s_adm, c) = adm;
-          AT(s_wait, c) = 0;
-          AT(s_nd, c) = d1;
-          peak_res = max(peak_res, cap - free_mem);
-          nk = ((t + d0) << 6) | c;
+  bool have = i < p.count, tdone = false, dmode = false;
+  uint32_t cur_t = 0;
+  if (have) { init(i); tdone = flags != 0; dmode = false; }  // static flags: no events
+  // Lanes advance through their traces independently but start and finish
+  // them together (warp vote below), so init/epilogue run converged.
+  while (__any_sync(kFull, have)) {
+    if (have && !tdone) {
+      uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
+      const uint32_t pf_lo = pfc_lo, pf_hi = pfc_hi;  // previous iteration's group
+      pfc_lo = 0; pfc_hi = 0;
+      if (!dmode) {
+        // ================= EVENT step (a2 + a3), branch-free =================
+        const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
+        const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
+        const uint32_t kmin = min(min(m01, m23), min(m45, m67));
+        if (kmin == kKeyNone) {
+          if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
+          tdone = true;
         } else {
-          const uint32_t cw = AT(s_cw, c);
+          const uint32_t t = kmin >> 6, c = kmin & 63u;
+          cur_t = t;
+          cp_wait1();  // every group but the previous iteration's is complete
+          if (bit64(pf_lo, pf_hi, c)) cp_wait0();
+          ++events;
+          const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
+          const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
+          const bool arr = (ust & kNotArrived) == kNotArrived;
           const uint32_t kind = cw >> 30, r = cw & kSizeMask, used = ust & kUsedMask;
-          bool adv = true;
-          if (kind == CONVGPU_OP_ALLOC) {
-            const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
-            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
-            if (need > L) {
-              ++n_rej;  // R10
-            } else if (need <= a) {
-              used_total += need - used;
-              peak_used = max(peak_used, used_total);
-              ust = (ust & ~kUsedMask) | need | kFirst;
-            } else {  // pause: reply withheld
-              ust |= kPaused;
-              AT(s_wait, c) -= t;
-              if (POLICY == CONVGPU_RECENT_FIT) AT(s_adm, c) = seq;
-              ++seq;
-              if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
-              adv = false;
-              disp = (target == kTargetNone);
+          const bool isA = !arr && kind == CONVGPU_OP_ALLOC;
+          const bool isF = !arr && kind == CONVGPU_OP_FREE;
+          const bool isX = !arr && kind == CONVGPU_OP_FINISH;
+          const bool tnone = target == kNoC, ctg = c == target;
+          const uint32_t a_c = (ust & kAdmitted) ? L : (ctg ? a_tg : 0u);
+          // ARRIVE (P:98, P:149 Fig. 3b/3c; R2)
+          const uint32_t g = (arr && tnone) ? min(L, free_mem) : 0u;
+          const bool vadm = arr && g == L;
+          const bool vtgt = arr && !vadm && g > 0;
+          // ALLOC
+          const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
+          const bool rej = isA && need > L;                // R10
+          const bool grant = isA && !rej && need <= a_c;
+          const bool pause = isA && !rej && !grant;       // reply withheld
+          // FREE (R11)
+          const bool badfree = isF && r > used;
+          // ledger
+          free_mem = free_mem - g + (isX ? a_c : 0u);
+          used_total = used_total + (grant ? need - used : 0u) - ((isF && !badfree) ? r : 0u) -
+                       (isX ? used : 0u);
+          peak_res = max(peak_res, cap - free_mem);
+          peak_used = max(peak_used, used_total);
+          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+          const bool clear_tg = isX && ctg;               // R20
+          target = vtgt ? c : (clear_tg ? kNoC : target);
+          a_tg = vtgt ? g : (clear_tg ? 0u : a_tg);
+          const uint32_t admv = (t << 6) | rank;
+          rank += vadm ? 1u : 0u;
+          n_rej += rej ? 1u : 0u;
+          live -= isX ? 1u : 0u;
+          if (pause) {
+            set64(pm_lo, pm_hi, c, true);
+            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(c, 0), true);
+            if (POLICY == CONVGPU_RECENT_FIT) {
+              if (sp < kStack) STK(sp) = (uint8_t)c;
+              ++sp;
+              ru_scan = ru_scan || sp > kStack;
+              AT(s_adm, c) = seq;  // suspension number (scan fallback)
             }
-          } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
-            if (r > used) {
-              flags |= CONVGPU_FLAG_INVALID_FREE;
-              adv = false;
-              done = true;
+            ++seq;
+          }
+          dmode = (pause && tnone) || isX;
+          if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true; }
+          const bool adv = !isX && !pause && !badfree;
+          // new state word
+          uint32_t nu = ust;
+          nu = grant ? ((ust & ~kUsedMask) | need | kFirst) : nu;
+          nu = (isF && !badfree) ? ust - r : nu;
+          nu = isX ? (ust & ~kUsedMask) : nu;
+          nu = pause ? (ust | kPaused) : nu;
+          nu = arr ? (vadm ? kAdmitted : 0u) : nu;
+          nu = (adv && !arr) ? nu + kKOne : nu;
+          AT(s_ust, c) = nu;
+          if (arr) AT(s_adm, c) = vadm ? admv : kKeyNone;
+          if (arr || isX) AT(s_nd, c) = arr ? am : t;     // d_1 / finish tick
+          kc = badfree ? kNoC : c;
+          nkc = adv ? (((t + nd) << 6) | c) : kKeyNone;
+          pfk = (adv && !arr) ? ((nu >> kKShift) & 7u) : 0xFFu;
+        }
+      } else {
+        // ====== one DISPATCH step at the triggering tick (R1, R9) ======
+        const uint32_t t = cur_t;
+        if (target != kNoC) {
+          const uint32_t tg = target;
+          const uint32_t Lt = AT(s_L, tg), ut = AT(s_ust, tg), cwt = AT(s_cw, tg),
+                         ndt = AT(s_nd, tg);
+          const uint32_t g = min(free_mem, Lt - a_tg);
+          a_tg += g;
+          free_mem -= g;
+          const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
+          const uint32_t uu = ut & kUsedMask;
+          const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
+          const bool full = a_tg == Lt;                          // admit, cascade
+          used_total += res ? pend : 0u;
+          peak_res = max(peak_res, cap - free_mem);
+          peak_used = max(peak_used, used_total);
+          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+          uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
+          nu |= full ? kAdmitted : 0u;
+          AT(s_ust, tg) = nu;
+          if (res) {
+            set64(pm_lo, pm_hi, tg, false);
+            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
+          }
+          if (full) AT(s_adm, tg) = (t << 6) | rank;
+          rank += full ? 1u : 0u;
+          target = full ? kNoC : target;
+          a_tg = full ? 0u : a_tg;
+          dmode = full;
+          kc = res ? tg : kNoC;
+          nkc = ((t + ndt) << 6) | tg;
+          pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
+        } else if (pm_lo | pm_hi) {
+          // ---- SELECT among paused ----
+          uint32_t sel;
+          if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
+            sel = ffs64(pm_lo, pm_hi);
+          } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
+            // R = #ranks with L <= free (limits sorted by (L, index))
+            uint32_t lo = 0, hi = n;
+#pragma unroll
+            for (int it = 0; it < 7; ++it) {
+              if (lo < hi) {
+                const uint32_t mid = (lo + hi) >> 1;
+                if (AT(s_ls, mid) <= free_mem) lo = mid + 1; else hi = mid;
+              }
+            }
+            uint32_t ml, mh;
+            lowmask64(lo, ml, mh);
+            const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
+            uint32_t rsel;
+            if (fl | fh) {  // largest fitting limit, lowest index among equals
+              const uint32_t h = fls64(fl, fh);
+              uint32_t gl, gh;
+              lowmask64(RKB(h, 1), gl, gh);
+              rsel = ffs64(pr_lo & ~gl, pr_hi & ~gh);
+            } else {  // smallest limit, lowest index
+              rsel = ffs64(pr_lo, pr_hi);
+            }
+            sel = RKB(rsel, 2);
+          } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5: most recent suspension
+            if (!ru_scan) {
+              while (sp > 0 && !bit64(pm_lo, pm_hi, STK(sp - 1))) --sp;  // lazy deletion
+              sel = STK(sp - 1);
             } else {
-              ust -= r;
-              used_total -= r;
-            }
-          } else if (kind == CONVGPU_OP_FINISH) {  // P:110, R18
-            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
-            free_mem += a;
-            used_total -= used;
-            ust &= ~kUsedMask;
-            AT(s_nd, c) = t;  // finish tick
-            --live;
-            if (c == target) { target = kTargetNone; a_tg = 0; }  // R20
-            adv = false;
-            disp = true;
-          }
-          if (adv) {
-            const uint32_t k = ((ust >> kKShift) & 7u) + 1u;
-            nk = ((t + AT(s_nd, c)) << 6) | c;
-            ust = (ust & ~kKMask) | (k << kKShift);
-            prefetch(c, k);
-          }
-        }
-        if (!done) {
-          AT(s_ust, c) = ust;
-          AT(s_key, c) = nk;
-          regroup(c);
-          // ---- DISPATCH (Fig. 3d; R1, R9) ----
-          if (disp) {
-            for (;;) {
-              if (target != kTargetNone) {
-                const uint32_t tg = target, Lt = AT(s_L, tg);
-                const uint32_t g = min(free_mem, Lt - a_tg);
-                a_tg += g;
-                free_mem -= g;
-                peak_res = max(peak_res, cap - free_mem);
-                uint32_t ut = AT(s_ust, tg);
-                if (ut & kPaused) {
-                  const uint32_t cwt = AT(s_cw, tg);
-                  const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
-                  const uint32_t uu = ut & kUsedMask;
-                  if (uu + pend <= a_tg) {  // RESUME (R9)
-                    used_total += pend;
-                    peak_used = max(peak_used, used_total);
-                    AT(s_wait, tg) += t;
-                    AT(s_adm, tg) = kKeyNone;
-                    if (tg < 32) pm_lo &= ~(1u << tg); else pm_hi &= ~(1u << (tg - 32));
-                    const uint32_t k = ((ut >> kKShift) & 7u) + 1u;
-                    ut = (ut & ~(kUsedMask | kKMask | kPaused)) | (uu + pend) | kFirst | (k << kKShift);
-                    AT(s_key, tg) = ((t + AT(s_nd, tg)) << 6) | tg;
-                    regroup(tg);
-                    prefetch(tg, k);
-                  }
-                }
-                if (a_tg == Lt) {  // fully guaranteed: admit, cascade leftover
-                  AT(s_adm, tg) = (t << 6) | rank; ++rank;
-                  AT(s_ust, tg) = ut | kAdmitted;
-                  target = kTargetNone;
-                  a_tg = 0;
-                  continue;
-                }
-                AT(s_ust, tg) = ut;
-                break;
-              }
-              if ((pm_lo | pm_hi) == 0u) break;
-              // ---- SELECT among paused ----
-              uint32_t sel;
-              if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
-                sel = pm_lo ? (uint32_t)(__ffs(pm_lo) - 1) : 32u + (uint32_t)(__ffs(pm_hi) - 1);
-              } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
-                uint32_t bf = kTargetNone, bfL = 0, bm = kTargetNone, bmL = 0;
+              uint32_t best = 0, bs = 0;
 #pragma unroll
-                for (uint32_t h = 0; h < 2; ++h) {
-                  uint32_t m = h ? pm_hi : pm_lo;
-                  while (m) {
-                    const uint32_t b = (uint32_t)(__ffs(m) - 1);
-                    m &= m - 1;
-                    const uint32_t cc = b + 32u * h;
-                    const uint32_t Lc = AT(s_L, cc);
-                    if (Lc <= free_mem && (bf == kTargetNone || Lc > bfL)) { bf = cc; bfL = Lc; }
-                    if (bm == kTargetNone || Lc < bmL) { bm = cc; bmL = Lc; }
-                  }
+              for (uint32_t h = 0; h < 2; ++h) {
+                uint32_t m = h ? pm_hi : pm_lo;
+                while (m) {
+                  const uint32_t b = (uint32_t)(__ffs(m) - 1);
+                  m &= m - 1;
+                  const uint32_t cc = b + 32u * h;
+                  const uint32_t sq = AT(s_adm, cc) + 1u;
+                  if (sq > bs) { bs = sq; best = cc; }
                 }
-                sel = (bf != kTargetNone) ? bf : bm;
-              } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
-                uint32_t best = 0, bs = 0;
-#pragma unroll
-                for (uint32_t h = 0; h < 2; ++h) {
-                  uint32_t m = h ? pm_hi : pm_lo;
-                  while (m) {
-                    const uint32_t b = (uint32_t)(__ffs(m) - 1);
-                    m &= m - 1;
-                    const uint32_t cc = b + 32u * h;
-                    const uint32_t sq = AT(s_adm, cc) + 1u;
-                    if (sq > bs) { bs = sq; best = cc; }
-                  }
-                }
-                sel = best;
-              } else {  // RANDOM_FIT (R6)
-                const uint64_t tid = p.tid_base + i;
-                const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
-                const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
-                                           (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
-                ++draws;
-                const uint32_t jj = __umulhi(x.x, m);
-                sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
               }
-              target = sel;
-              a_tg = 0;
-              ++n_sel;
+              sel = best;
             }
+          } else {  // RANDOM_FIT (R6)
+            const uint64_t tid = p.tid_base + i;
+            const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
+            const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                       (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+            ++draws;
+            const uint32_t jj = __umulhi(x.x, m);
+            sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
           }
-          if (used_total > cap - free_mem || free_mem > cap) flags |= CONVGPU_FLAG_OVERCOMMIT;
+          target = sel;
+          a_tg = 0;
+          ++n_sel;
+        } else {
+          dmode = false;
         }
-        cp_commit();
       }
+      // ---- shared tail: key update, group re-min, op prefetch ----
+      if (kc != kNoC) {
+        AT(s_key, kc) = nkc;
+        regroup(kc);
+        if (pfk != 0xFFu) {  // op k word, delta of op k+1
+          if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + (size_t)pfk * n + kc);
+          if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + (size_t)(pfk + 1) * n + kc);
+          set64(pfc_lo, pfc_hi, kc, true);
+        }
+      }
+      cp_commit();
     }
-    if (done) {
+    if (__all_sync(kFull, !have || tdone) && have) {
       epilogue(i);
       i += T;
       have = i < p.count;
-      if (have) { init(i); halted = flags != 0; }
+      if (have) { init(i); tdone = flags != 0; dmode = false; }
     }
   }
+#undef STK
+#undef RKB
 #undef AT
 
   // ---- statistics: warp -> grid (a6) ----
@@ -436,31 +503,29 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   }
 }
 
-template <int POLICY, int MODE>
-static cudaError_t launch_m(const ReplayArgs& a, cudaStream_t stream) {
-  const size_t smem = (size_t)(kLptThreads / 32) * warp_bytes(a.n);
-  auto kern = replay_lpt_kernel<POLICY, MODE>;
+template <int POLICY>
+static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
+  // Best-Fit's rank tables make a warp's slice 64 KB: one warp per CTA packs
+  // three per SM; the others fit two 2-warp CTAs (four warps) per SM.
+  const int threads = POLICY == CONVGPU_BEST_FIT ? 32 : kLptThreads;
+  const size_t smem = (size_t)(threads / 32) * warp_bytes(POLICY, a.n);
+  auto kern = replay_lpt_kernel<POLICY>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0, per_sm = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
-  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kLptThreads, smem)) !=
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem)) !=
       cudaSuccess)
     return e;
   if (per_sm < 1) return cudaErrorInvalidConfiguration;
-  const uint64_t need = (a.count + kLptThreads - 1) / kLptThreads;
+  const uint64_t need = (a.count + threads - 1) / threads;
   uint64_t grid = (uint64_t)sms * (uint64_t)per_sm;
   if (a.grid_override) grid = a.grid_override;
   if (grid > need) grid = need;
   if (grid < 1) grid = 1;
-  kern<<<(unsigned)grid, kLptThreads, smem, stream>>>(a);
+  kern<<<(unsigned)grid, threads, smem, stream>>>(a);
   return cudaGetLastError();
-}
-
-template <int POLICY>
-static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
-  return launch_m<POLICY, 0>(a, stream);
 }
 
 }  // namespace lpt
