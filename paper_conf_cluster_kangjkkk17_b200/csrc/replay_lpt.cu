@@ -96,11 +96,13 @@ __device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi
   hi = r >= 64 ? 0xFFFFFFFFu : (r <= 32 ? 0u : ((1u << (r - 32)) - 1u));
 }
 
-template <int POLICY>
+// NF, KF: compile-time container / op counts (64, 4 for the configs) or 0.
+template <int POLICY, int NF, int KF>
 __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
   const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
-  const uint32_t n = p.n, K = p.K, cap = p.cap, ovh = p.ovh;
+  const uint32_t n = NF ? (uint32_t)NF : p.n, K = KF ? (uint32_t)KF : p.K;
+  const uint32_t cap = p.cap, ovh = p.ovh;
   uint32_t* const W0 = smem_w + (wib * warp_bytes(POLICY, n)) / 4;
   uint32_t* const S = W0 + lane;
   uint32_t* const s_key = S + (size_t)W_KEY * n * 32;
@@ -503,13 +505,13 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   }
 }
 
-template <int POLICY>
+template <int POLICY, int NF, int KF>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
   // Best-Fit's rank tables make a warp's slice 64 KB: one warp per CTA packs
   // three per SM; the others fit two 2-warp CTAs (four warps) per SM.
   const int threads = POLICY == CONVGPU_BEST_FIT ? 32 : kLptThreads;
   const size_t smem = (size_t)(threads / 32) * warp_bytes(POLICY, a.n);
-  auto kern = replay_lpt_kernel<POLICY>;
+  auto kern = replay_lpt_kernel<POLICY, NF, KF>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0, per_sm = 0;
@@ -530,12 +532,18 @@ static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
 
 }  // namespace lpt
 
+template <int POLICY>
+static cudaError_t launch_p(const ReplayArgs& a, cudaStream_t stream) {
+  if (a.n == 64 && a.K == 4) return lpt::launch_t<POLICY, 64, 4>(a, stream);
+  return lpt::launch_t<POLICY, 0, 0>(a, stream);
+}
+
 cudaError_t launch_replay_lpt(const ReplayArgs& a, int policy, cudaStream_t stream) {
   switch (policy) {
-    case CONVGPU_FIFO: return lpt::launch_t<CONVGPU_FIFO>(a, stream);
-    case CONVGPU_BEST_FIT: return lpt::launch_t<CONVGPU_BEST_FIT>(a, stream);
-    case CONVGPU_RECENT_FIT: return lpt::launch_t<CONVGPU_RECENT_FIT>(a, stream);
-    case CONVGPU_RANDOM_FIT: return lpt::launch_t<CONVGPU_RANDOM_FIT>(a, stream);
+    case CONVGPU_FIFO: return launch_p<CONVGPU_FIFO>(a, stream);
+    case CONVGPU_BEST_FIT: return launch_p<CONVGPU_BEST_FIT>(a, stream);
+    case CONVGPU_RECENT_FIT: return launch_p<CONVGPU_RECENT_FIT>(a, stream);
+    case CONVGPU_RANDOM_FIT: return launch_p<CONVGPU_RANDOM_FIT>(a, stream);
   }
   return cudaErrorInvalidValue;
 }
