@@ -336,7 +336,9 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             }
             ++seq;
           }
-          dmode = (pause && tnone) || isX;
+          // DISPATCH has work after a pause with no target (select) or a
+          // FINISH that leaves a target to fill or paused containers
+          dmode = (pause && tnone) || (isX && (target != kNoC || (pm_lo | pm_hi) != 0u));
           if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true; }
           const bool adv = !isX && !pause && !badfree;
           // new state word
@@ -356,39 +358,12 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
         }
       } else {
         // ====== one DISPATCH step at the triggering tick (R1, R9) ======
+        // A step = [SELECT if there is no fill target] + fill / resume / admit
+        // of the target; an admit keeps the lane in dispatch mode (the
+        // leftover cascades to the next selection, Fig. 3d).
         const uint32_t t = cur_t;
-        if (target != kNoC) {
-          const uint32_t tg = target;
-          const uint32_t Lt = AT(s_L, tg), ut = AT(s_ust, tg), cwt = AT(s_cw, tg),
-                         ndt = AT(s_nd, tg);
-          const uint32_t g = min(free_mem, Lt - a_tg);
-          a_tg += g;
-          free_mem -= g;
-          const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
-          const uint32_t uu = ut & kUsedMask;
-          const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
-          const bool full = a_tg == Lt;                          // admit, cascade
-          used_total += res ? pend : 0u;
-          peak_res = max(peak_res, cap - free_mem);
-          peak_used = max(peak_used, used_total);
-          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
-          uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
-          nu |= full ? kAdmitted : 0u;
-          AT(s_ust, tg) = nu;
-          if (res) {
-            set64(pm_lo, pm_hi, tg, false);
-            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
-          }
-          if (full) AT(s_adm, tg) = (t << 6) | rank;
-          rank += full ? 1u : 0u;
-          target = full ? kNoC : target;
-          a_tg = full ? 0u : a_tg;
-          dmode = full;
-          kc = res ? tg : kNoC;
-          nkc = ((t + ndt) << 6) | tg;
-          pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
-        } else if (pm_lo | pm_hi) {
-          // ---- SELECT among paused ----
+        if (target == kNoC) {
+          // ---- SELECT among paused; pm != 0 here ----
           uint32_t sel;
           if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
             sel = ffs64(pm_lo, pm_hi);
@@ -446,8 +421,37 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           target = sel;
           a_tg = 0;
           ++n_sel;
-        } else {
-          dmode = false;
+        }
+        {
+          const uint32_t tg = target;
+          const uint32_t Lt = AT(s_L, tg), ut = AT(s_ust, tg), cwt = AT(s_cw, tg),
+                         ndt = AT(s_nd, tg);
+          const uint32_t g = min(free_mem, Lt - a_tg);
+          a_tg += g;
+          free_mem -= g;
+          const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
+          const uint32_t uu = ut & kUsedMask;
+          const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
+          const bool full = a_tg == Lt;                          // admit, cascade
+          used_total += res ? pend : 0u;
+          peak_res = max(peak_res, cap - free_mem);
+          peak_used = max(peak_used, used_total);
+          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+          uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
+          nu |= full ? kAdmitted : 0u;
+          AT(s_ust, tg) = nu;
+          if (res) {
+            set64(pm_lo, pm_hi, tg, false);
+            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
+          }
+          if (full) AT(s_adm, tg) = (t << 6) | rank;
+          rank += full ? 1u : 0u;
+          target = full ? kNoC : target;
+          a_tg = full ? 0u : a_tg;
+          dmode = full && (pm_lo | pm_hi) != 0u;  // another selection follows
+          kc = res ? tg : kNoC;
+          nkc = ((t + ndt) << 6) | tg;
+          pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
         }
       }
       // ---- shared tail: key update, group re-min, op prefetch ----
