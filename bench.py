@@ -269,7 +269,7 @@ def run_ours(args, rank, local_rank, world):
     def kernel_of(p):  # the rule of abi.cu auto_variant
         if args.kernel != "auto":
             return args.kernel
-        return "lane" if Nr >= sms * 2 * 64 * 4 and p != "best_fit" else "warp"
+        return "lane" if Nr >= sms * 2 * 64 * 4 else "warp"
     kernel_used = ",".join(sorted({kernel_of(p) for p in POLICIES}))
     # correctness of the timed work: every timed launch replayed every trace
     last = args.warmup + args.steps - 1

@@ -79,15 +79,15 @@ bool use_bulk(const convgpu::ReplayArgs& a) {
 }
 
 // Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, profiles/):
-// lane-per-trace needs enough traces to give every SM several CTAs; it wins
-// for FIFO, Recent-Fit and Random-Fit.  Best-Fit's per-trace rank tables cost
-// occupancy and an O(n^2) init there, so it stays on warp-per-trace.
+// lane-per-trace keeps 32 traces per warp in flight and needs enough traces
+// to give every SM several CTAs; below that warp-per-trace keeps more SMs
+// busy.  (policy is accepted for per-policy tuning; all four currently agree.)
 uint32_t auto_variant(uint64_t count, int policy) {
+  (void)policy;
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const bool big = count >= (uint64_t)sms * 2 * convgpu::kLptThreads * 4;
-  const bool o1 = policy != CONVGPU_BEST_FIT;
-  return (big && o1) ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
+  return big ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
 }
 
 cudaError_t launch_any(const convgpu::ReplayArgs& a, int policy, uint32_t variant, cudaStream_t s) {

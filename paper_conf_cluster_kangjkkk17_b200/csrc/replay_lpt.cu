@@ -183,19 +183,53 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     if (POLICY == CONVGPU_BEST_FIT) {
       // ranks of (L, index) ascending; gs = first rank with the same L
-      for (uint32_t c = 0; c < n; ++c) {
-        const uint32_t Lc = AT(s_L, c);
-        uint32_t lt = 0, eq = 0;
-        for (uint32_t d = 0; d < n; ++d) {
-          const uint32_t Ld = AT(s_L, d);
-          lt += (Ld < Lc) ? 1u : 0u;
-          eq += (Ld == Lc && d < c) ? 1u : 0u;
+      if (NF == 64) {
+        // bitonic sort network over the 64 packed keys L << 6 | c (L < 2^26)
+        uint32_t v[64];
+#pragma unroll
+        for (int c = 0; c < 64; ++c) v[c] = (AT(s_L, c) << 6) | (uint32_t)c;
+#pragma unroll
+        for (int k = 2; k <= 64; k <<= 1) {
+#pragma unroll
+          for (int j = k >> 1; j > 0; j >>= 1) {
+#pragma unroll
+            for (int x = 0; x < 64; ++x) {
+              const int y = x ^ j;
+              if (y > x) {
+                const uint32_t a = v[x], b = v[y];
+                const bool up = (x & k) == 0;
+                v[x] = up ? min(a, b) : max(a, b);
+                v[y] = up ? max(a, b) : min(a, b);
+              }
+            }
+          }
         }
-        const uint32_t r = lt + eq;
-        RKB(c, 0) = (uint8_t)r;
-        RKB(r, 1) = (uint8_t)lt;
-        RKB(r, 2) = (uint8_t)c;
-        AT(s_ls, r) = Lc;
+        uint32_t gsr = 0, prevL = 0xFFFFFFFFu;
+#pragma unroll
+        for (int r = 0; r < 64; ++r) {
+          const uint32_t c = v[r] & 63u, Lc = v[r] >> 6;
+          gsr = (Lc == prevL) ? gsr : (uint32_t)r;
+          prevL = Lc;
+          RKB(c, 0) = (uint8_t)r;
+          RKB(r, 1) = (uint8_t)gsr;
+          RKB(r, 2) = (uint8_t)c;
+          AT(s_ls, r) = Lc;
+        }
+      } else {
+        for (uint32_t c = 0; c < n; ++c) {
+          const uint32_t Lc = AT(s_L, c);
+          uint32_t lt = 0, eq = 0;
+          for (uint32_t d = 0; d < n; ++d) {
+            const uint32_t Ld = AT(s_L, d);
+            lt += (Ld < Lc) ? 1u : 0u;
+            eq += (Ld == Lc && d < c) ? 1u : 0u;
+          }
+          const uint32_t r = lt + eq;
+          RKB(c, 0) = (uint8_t)r;
+          RKB(r, 1) = (uint8_t)lt;
+          RKB(r, 2) = (uint8_t)c;
+          AT(s_ls, r) = Lc;
+        }
       }
     }
     flags = bad;
