@@ -107,6 +107,9 @@ def _p(a, ct=C.c_uint32):
     return None if a is None else a.ctypes.data_as(C.POINTER(ct))
 
 
+LITERAL = 0x100  # OR into the policy: literal re-select-on-every-release reading
+
+
 def _pol(policy) -> int:
     return POLICY[policy] if isinstance(policy, str) else int(policy)
 

@@ -49,8 +49,9 @@ class Violation(AssertionError):
 class _S:
     """Scheduler state for one path."""
 
-    def __init__(self, tr, cap, ovh):
+    def __init__(self, tr, cap, ovh, lit=False):
         n = len(tr["arrival"])
+        self.lit = lit
         self.n = n
         self.cap = cap
         self.ovh = ovh
@@ -91,6 +92,11 @@ def _checks(s, tr):
         raise Violation("capacity ledger")
     if sum(s.used) > s.cap:
         raise Violation("memory in use exceeds capacity")
+    if s.lit:  # the literal reading keeps partial holds: only the ledger checks apply
+        for c in range(s.n):
+            if not (0 <= s.used[c] <= s.a[c] <= L[c]):
+                raise Violation("used <= a <= L")
+        return
     partial = [c for c in range(s.n) if s.state[c] == "live" and 0 < s.a[c] < L[c]]
     if len(partial) > 1 or (partial and partial[0] != s.target):
         raise Violation("more than one partially assigned container")
@@ -123,12 +129,12 @@ def _apply(s, tr, c, t):
     L = tr["limit"][c]
     if s.state[c] == "pending":
         s.state[c] = "live"
-        g = min(L, s.free) if s.target is None else 0
+        g = min(L, s.free) if (s.lit or s.target is None) else 0
         s.a[c] = g
         s.free -= g
         if g == L:
             _admit(s, c, t)
-        elif g > 0:
+        elif g > 0 and not s.lit:
             s.target = c
         s.nt[c] = t + tr["delta"][0][c]
         return
@@ -187,8 +193,38 @@ def _rule_picks(s, tr, tid, seed):
     return P, picks
 
 
+def _dispatch_lit(s, tr, t, tid, seed):
+    """Literal reading (R1-LIT): while memory is free and someone is paused,
+    ANY paused container may be chosen; it receives min(free, L - a)."""
+    L = tr["limit"]
+    if s.free == 0 or not any(s.paused):
+        yield s
+        return
+    P, picks = _rule_picks(s, tr, tid, seed)
+    for i, c in enumerate(P):
+        s2 = copy.deepcopy(s) if i < len(P) - 1 else s
+        s2.obeys = {p for p in s2.obeys if picks[p] == c}
+        s2.choices.append(("select", c, tuple(P)))
+        s2.nsel += 1
+        g = min(s2.free, L[c] - s2.a[c])
+        s2.a[c] += g
+        s2.free -= g
+        if s2.paused[c] and s2.used[c] + s2.pend[c] <= s2.a[c]:
+            s2.used[c] += s2.pend[c]
+            s2.first[c] = True
+            s2.paused[c] = False
+            s2.wait[c] += t - s2.stick[c]
+            _advance(s2, tr, c, t)
+        if s2.a[c] == L[c]:
+            _admit(s2, c, t)
+        yield from _dispatch_lit(s2, tr, t, tid, seed)
+
+
 def _dispatch(s, tr, t, tid, seed):
     """Yield every state reachable by DISPATCH, branching on selections."""
+    if s.lit:
+        yield from _dispatch_lit(s, tr, t, tid, seed)
+        return
     L = tr["limit"]
     while True:
         if s.target is not None:
@@ -236,7 +272,9 @@ def _run(s, tr, tid, seed, permute_ties):
         if not cands:
             if any(st != "done" for st in s.state):
                 s.flags |= 1
-                raise Violation("deadlock: containers remain but none can run")
+                if not s.lit:
+                    raise Violation("deadlock: containers remain but none can run")
+                s.stopped = True
             yield s
             return
         cands.sort()
@@ -271,7 +309,7 @@ def outcome(s, tr):
                 n_rejected=s.nrej, n_select=s.nsel, flags=s.flags)
 
 
-def explore(tr, cap, ovh=0, tid=0, seed=0, permute_ties=False, max_paths=200000):
+def explore(tr, cap, ovh=0, tid=0, seed=0, permute_ties=False, max_paths=200000, lit=False):
     """Return a list of (outcome, obeyed_policies, canonical, choices) per path.
 
     tr: dict(arrival=[n], limit=[n], delta=[K][n], arg=[K][n]) of Python ints.
@@ -280,7 +318,7 @@ def explore(tr, cap, ovh=0, tid=0, seed=0, permute_ties=False, max_paths=200000)
     tr = {k: [list(map(int, r)) for r in v] if k in ("delta", "arg") else list(map(int, v))
           for k, v in tr.items() if k in ("arrival", "limit", "delta", "arg")}
     paths = []
-    for s in _run(_S(tr, cap, ovh), tr, tid, seed, permute_ties):
+    for s in _run(_S(tr, cap, ovh, lit), tr, tid, seed, permute_ties):
         paths.append((outcome(s, tr), frozenset(s.obeys), s.canonical, tuple(s.choices)))
         if len(paths) > max_paths:
             raise RuntimeError("path explosion")

@@ -89,6 +89,7 @@ typedef struct {
   uint64_t events;
   int stop;
   int check;
+  int lit; /* 1 = literal re-select-on-every-release reading (NEXT-1, R1-LIT) */
   int32_t violation;
   uint64_t violation_event;
 } sim_t;
@@ -128,12 +129,13 @@ static void ev_arrive(sim_t *s, int c, uint32_t t) {
   uint32_t L = L_of(s, c);
   x->st = ST_LIVE;
   uint32_t g = 0;
-  if (s->target < 0) g = (L < s->free_mem) ? L : s->free_mem;
+  /* R1-LIT: without a sticky target every newcomer takes what is free */
+  if (s->lit || s->target < 0) g = (L < s->free_mem) ? L : s->free_mem;
   x->a = g;
   s->free_mem -= g;
   if (g == L)
     admit(s, c, t);
-  else if (g > 0)
+  else if (g > 0 && !s->lit)
     s->target = c;
   x->next_tick = t + delta_of(s, c, 0);
 }
@@ -251,7 +253,48 @@ static int select_paused(sim_t *s) {
  * its memory and resumes; the remainder goes to D, which stays suspended).
  * Reading R1 (sticky fill target), R9 (resume as soon as the withheld
  * request is covered), R16 (runs after every event). */
+static void resume_if_covered(sim_t *s, int c, uint32_t t);
+
+/* DISPATCH under the literal reading R1-LIT: every
+ * time memory is free and someone is paused, the policy picks a paused
+ * container (shortfall L - a counting partial holds) and
+ * assigns it min(free, L - a); partial assignments are kept; the loop goes
+ * on while memory is left.  Nothing guarantees progress, so this reading
+ * can deadlock (R1). */
+static void dispatch_lit(sim_t *s, uint32_t t) {
+  for (;;) {
+    if (s->free_mem == 0) break;
+    int any_paused = 0;
+    for (uint32_t c = 0; c < s->tr->n; ++c) any_paused |= s->c[c].paused;
+    if (!any_paused) break;
+    int x = select_paused(s);
+    s->n_select++;
+    cont_t *y = &s->c[x];
+    uint32_t room = L_of(s, x) - y->a;
+    uint32_t g = (s->free_mem < room) ? s->free_mem : room;
+    y->a += g;
+    s->free_mem -= g;
+    resume_if_covered(s, x, t);
+    if (y->a == L_of(s, x)) admit(s, x, t);
+  }
+}
+
+static void resume_if_covered(sim_t *s, int c, uint32_t t) {
+  cont_t *x = &s->c[c];
+  if (x->paused && (uint64_t)x->used + x->pending <= x->a) { /* RESUME (R9) */
+    x->used += x->pending;
+    x->first_done = 1;
+    x->paused = 0;
+    x->wait += t - x->susp_tick;
+    advance(s, c, t);
+  }
+}
+
 static void dispatch(sim_t *s, uint32_t t) {
+  if (s->lit) {
+    dispatch_lit(s, t);
+    return;
+  }
   for (;;) {
     if (s->target >= 0) {
       int tg = s->target;
@@ -299,12 +342,13 @@ static int check_invariants(const sim_t *s) {
     if (x->st == ST_LIVE && x->admitted && x->a != L) return 5; /* admitted => full */
     if (x->st == ST_LIVE && x->a > 0 && x->a < L) {
       partial++;
-      if ((int)c != s->target) return 6;     /* partial => it is the target */
+      if (!s->lit && (int)c != s->target) return 6; /* partial => it is the target */
     }
     if (x->paused && x->st != ST_LIVE) return 7;
-    if (x->paused && s->target < 0) return 8; /* NONE => none paused */
+    if (!s->lit && x->paused && s->target < 0) return 8; /* NONE => none paused */
   }
   if (sum_a + s->free_mem != s->cap) return 1; /* ledger conserves capacity */
+  if (s->lit) return 0;
   if (partial > 1) return 9;
   if (s->target >= 0 && s->free_mem != 0) return 10;
   if (s->target >= 0 && s->c[s->target].st != ST_LIVE) return 11;
@@ -341,10 +385,12 @@ static uint32_t static_flags(const orc_trace_t *tr, uint32_t cap) {
   return f;
 }
 
-int orc_replay(const orc_trace_t *tr, uint32_t cap, int policy, uint64_t tid,
+int orc_replay(const orc_trace_t *tr, uint32_t cap, int policy_mode, uint64_t tid,
                uint64_t rand_seed, uint32_t ovh, int check, orc_result_t *res) {
+  const int policy = policy_mode & 0xFF, lit = (policy_mode & ORC_LITERAL) != 0;
   if (!tr || !res || tr->n < 1 || tr->n > ORC_MAX_N || tr->K < 1 ||
-      tr->K > ORC_MAX_K || policy < 0 || policy > 3 || cap == 0)
+      tr->K > ORC_MAX_K || policy < 0 || policy > 3 || (policy_mode & ~(0xFF | ORC_LITERAL)) ||
+      cap == 0)
     return -1;
   sim_t *s = (sim_t *)calloc(1, sizeof(sim_t));
   if (!s) return -2;
@@ -357,6 +403,7 @@ int orc_replay(const orc_trace_t *tr, uint32_t cap, int policy, uint64_t tid,
   s->free_mem = cap;
   s->target = -1;
   s->check = check;
+  s->lit = lit;
   for (uint32_t c = 0; c < tr->n; ++c) {
     s->c[c].st = ST_PENDING;
     s->c[c].admit_tick = ORC_NONE32;

@@ -24,6 +24,10 @@ extern "C" {
 /* Scheduling policies. */
 enum { ORC_FIFO = 0, ORC_BEST_FIT = 1, ORC_RECENT = 2, ORC_RANDOM = 3 };
 
+/* Dispatch-reading flag OR-ed into the policy argument: the literal
+ * re-select-on-every-release reading (R1-LIT). */
+#define ORC_LITERAL 0x100
+
 /* Op kinds carried in the top two bits of an op word; low 30 bits = MiB. */
 enum { ORC_ALLOC = 0, ORC_FREE = 1, ORC_FINISH = 2, ORC_NOP = 3 };
 

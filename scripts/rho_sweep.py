@@ -1,0 +1,101 @@
+#!/usr/bin/env python
+"""BASELINE config [4]: capacity / oversubscription sweep on the 180 GiB model.
+
+For rho = 1..8 (declared limits scaled by 15*rho/7, so E[sum L]/cap = rho),
+10^6 traces x 64 containers per point, Random-Fit replayed with seeds
+0..31 and FIFO / Best-Fit / Recent-Fit once, all on the GPU through the C ABI
+(statistics only, no per-trace outputs).  Writes per-(rho, policy, seed) means
+and the seed spread to profiles/<tag>_rho_sweep.json and a markdown table.
+
+  python scripts/rho_sweep.py [--traces 1000000] [--seeds 32] [--tag r01]
+
+Sharding over G GPUs (torchrun) splits each point's trace-id range; on one GPU
+the points run back to back.  Parity of the sweep's kernels against the
+oracle is covered by tests/test_gpu_parity.py::test_rho_sweep_window.
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--traces", type=int, default=1_000_000)
+    ap.add_argument("--seeds", type=int, default=32)
+    ap.add_argument("--tag", default="r01")
+    a = ap.parse_args()
+    import torch
+
+    import paper_conf_cluster_kangjkkk17_b200 as cg
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    rows = []
+    t_all = time.time()
+    buf = None
+    for rho in range(1, 9):
+        w = W.rho_sweep(rho, n_traces=a.traces)
+        buf = cg.generate(w.gen, 0, a.traces, device=dev, out=buf)
+        runs = [("fifo", 0), ("best_fit", 0), ("recent_fit", 0)] + \
+               [("random_fit", s) for s in range(a.seeds)]
+        for pol, seed in runs:
+            out = cg.alloc_out(a.traces, w.gen.n, device=dev, full=False, summary=False)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            cg.replay(buf, w.cap, pol, out, rand_seed=seed)
+            e1.record()
+            torch.cuda.synchronize()
+            st = cg.stats_dict(out.stats_np())
+            assert st["traces"] == a.traces
+            rows.append({"rho": rho, "policy": pol, "seed": seed,
+                         "mean_makespan_s": st["sum_makespan"] / st["traces"] / 1000.0,
+                         "mean_wait_s": st["sum_wait"] / (st["traces"] * w.gen.n) / 1000.0,
+                         "selections_per_trace": st["n_select"] / st["traces"],
+                         "max_peak_reserved_mib": st["max_peak_reserved"],
+                         "flag_count": st["flag_count"], "digest_sum": "%016x" % st["digest_sum"],
+                         "events": st["events"], "ms": e0.elapsed_time(e1)})
+    table = []
+    for rho in range(1, 9):
+        line = {"rho": rho}
+        for pol in ("fifo", "best_fit", "recent_fit"):
+            r = [x for x in rows if x["rho"] == rho and x["policy"] == pol][0]
+            line[pol] = (r["mean_makespan_s"], r["mean_wait_s"])
+        rr = [x for x in rows if x["rho"] == rho and x["policy"] == "random_fit"]
+        mk = [x["mean_makespan_s"] for x in rr]
+        wt = [x["mean_wait_s"] for x in rr]
+        line["random_fit"] = {"makespan_mean": statistics.mean(mk),
+                              "makespan_sd": statistics.pstdev(mk),
+                              "makespan_min": min(mk), "makespan_max": max(mk),
+                              "wait_mean": statistics.mean(wt), "wait_sd": statistics.pstdev(wt)}
+        line["deadlocks"] = sum(x["flag_count"][0] for x in rows if x["rho"] == rho)
+        table.append(line)
+    ev = sum(x["events"] for x in rows)
+    ms = sum(x["ms"] for x in rows)
+    doc = {"config": "BASELINE configs[4]", "traces_per_point": a.traces, "seeds": a.seeds,
+           "capacity_mib": 184320, "containers": 64, "unit_time": "s (1 tick = 1 ms)",
+           "replay_events": ev, "replay_ms": ms, "events_per_s": ev / (ms / 1e3),
+           "wall_s": time.time() - t_all, "table": table, "runs": rows}
+    os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
+    with open(os.path.join(ROOT, "gpurun_out", f"{a.tag}_rho_sweep.json")
+              if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else
+              os.path.join(ROOT, "profiles", f"{a.tag}_rho_sweep.json"), "w") as f:
+        json.dump(doc, f, indent=1)
+    print("rho | FIFO makespan/wait | BF | RU | Rand makespan mean±sd [min,max] / wait | deadlocks")
+    for l in table:
+        r = l["random_fit"]
+        print(f"{l['rho']} | {l['fifo'][0]:.1f}/{l['fifo'][1]:.1f} | {l['best_fit'][0]:.1f}/"
+              f"{l['best_fit'][1]:.1f} | {l['recent_fit'][0]:.1f}/{l['recent_fit'][1]:.1f} | "
+              f"{r['makespan_mean']:.2f}±{r['makespan_sd']:.3f} [{r['makespan_min']:.2f},"
+              f"{r['makespan_max']:.2f}] / {r['wait_mean']:.2f} | {l['deadlocks']}")
+    print(f"{ev:.3e} events in {ms / 1e3:.2f} s of replay = {ev / (ms / 1e3):.3e} events/s")
+
+
+if __name__ == "__main__":
+    main()

@@ -76,3 +76,27 @@ def test_same_tick_interleavings_n4(orc):
     b = W.random_batch(5, 40, 4, 3, 8, mode="delayed", max_arrival_step=2,
                        limit_choices=range(1, 9))
     _check_batch(orc, b, 8, 0, permute=True, max_paths=50000)
+
+
+@pytest.mark.parametrize("mode", ["valid", "delayed", "over"])
+def test_literal_reading_policy_paths_match_oracle(orc, mode):
+    """R1-LIT (NEXT-1): the explorer's literal dispatch (any paused container
+    at every release, partial holds kept) contains the oracle's answer for
+    each policy as the canonical path obeying that policy's rule; deadlocks
+    are outcomes here, not violations."""
+    b = W.random_batch(7, 200, 4, 3, 8, mode=mode, max_arrival_step=1,
+                       limit_choices=range(1, 9))
+    dead = 0
+    for i in range(b.count):
+        tr = dict(arrival=b.arrival[i], limit=b.limit[i], delta=b.delta[i], arg=b.arg[i])
+        paths = B.explore(tr, 8, tid=i, seed=3, lit=True)
+        dead += any(o["flags"] & 1 for o, _, _, _ in paths)
+        for k, p in enumerate(POLS):
+            r = orc.replay_trace(tr["arrival"], tr["limit"], tr["delta"], tr["arg"], 8,
+                                 k | 0x100, tid=i, seed=3)
+            assert r["violation"] == 0
+            cand = [o for o, ob, can, _ in paths if p in ob and can]
+            assert len(cand) == 1
+            for key in KEYS:
+                assert cand[0][key] == r[key], (i, p, key)
+    assert dead > 0  # the literal reading admits deadlocking schedules

@@ -170,12 +170,12 @@ def test_mimic_with_overhead(cg, orc, kernel, policy):
 
 
 @pytest.mark.parametrize("policy", POLS)
-@pytest.mark.parametrize("rho", [1, 4, 8])
+@pytest.mark.parametrize("rho", [1, 2, 3, 4, 5, 6, 7, 8])
 @pytest.mark.parametrize("kernel", KERNELS)
 def test_rho_sweep_window(cg, orc, kernel, policy, rho):
     w = W.rho_sweep(rho, rand_seed=rho * 7 + 1)
-    ref = orc.replay_range(w, policy, 10_000, 11_500, full=True)
-    tr = cg.generate(w.gen, 10_000, 1_500)
+    ref = orc.replay_range(w, policy, 10_000, 11_000, full=True)
+    tr = cg.generate(w.gen, 10_000, 1_000)
     out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel=kernel)
     _compare(cg, out, ref)
 

@@ -321,3 +321,55 @@ def test_generator_recipe(orc):
             assert sizes[0] + sizes[1] == L[c] and sizes[2] == sizes[0]
     exp = counts.sum() / 6
     assert float(((counts - exp) ** 2 / exp).sum()) < 20.5  # p=0.001, 5 dof
+
+
+# --- NEXT-1: the literal re-select-on-every-release reading (R1-LIT) -------
+LIT = 0x100
+
+
+def _survey_counterexample():
+    """cap 20; G (L 10) and F (L 4) run from t=0, G
+    exits at t=2, F at t=100; X (L 20) arrives at t=1 and Z (L 18) at t=3,
+    both ALLOC their whole limit at t=50 and run 10 more ticks."""
+    arrival = np.array([0, 0, 1, 3], np.uint32)
+    limit = np.array([10, 4, 20, 18], np.uint32)
+    delta = np.array([[0, 0, 49, 47], [2, 100, 10, 10]], np.uint32)
+    arg = np.array([[op(ALLOC, 10), op(ALLOC, 4), op(ALLOC, 20), op(ALLOC, 18)],
+                    [op(FINISH)] * 4], np.uint32)
+    return arrival, limit, delta, arg
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_literal_reading_deadlocks_where_sticky_does_not(orc, policy):
+    """P:7 claims the policies prevent deadlock.  Under R1 (sticky target) the
+    counterexample completes; under the literal reading every policy leaves X
+    and Z paused on partial holds that can never be completed."""
+    a, L, d, g = _survey_counterexample()
+    r = orc.replay_trace(a, L, d, g, 20, policy)
+    assert r["flags"] == 0 and r["finish"][2] > 0 and r["finish"][3] > 0
+    rl = orc.replay_trace(a, L, d, g, 20, POLS.index(policy) | LIT)
+    assert rl["flags"] == 1 and rl["violation"] == 0  # DEADLOCK, ledger intact
+
+
+def test_literal_reading_contradicts_fig3_for_best_fit(orc):
+    """Under the literal reading Best-Fit gives B's 3072 MiB to D (the closest
+    fit) at t=50, not to C as Fig. 3d narrates — one reason DESIGN.md
+    takes the sticky reading R1."""
+    f = W.fig3_fixture()
+    r = orc.replay_trace(f["arrival"], f["limit"], f["delta"], f["arg"], f["cap"], 1 | LIT)
+    assert r["admit_tick"][3] == 50 and r["admit_tick"][2] != 50
+    r = orc.replay_trace(f["arrival"], f["limit"], f["delta"], f["arg"], f["cap"], 0 | LIT)
+    assert r["admit_tick"] == [0, 0, 50, 150]  # FIFO happens to agree
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_literal_reading_invariants_and_deadlock_rate(orc, policy):
+    """The ledger invariants still hold under the literal reading; on the
+    paper-mimic workload (one container every 5 s) it deadlocks a
+    share of traces that the sticky reading completes."""
+    w = W.CONFIGS["mimic"]
+    sticky = orc.replay_range(w, policy, 0, 200, check=True)
+    lit = orc.replay_range(w, POLS.index(policy) | LIT, 0, 200, check=True)
+    assert sticky["rc"] == 0 and lit["rc"] == 0
+    assert sticky["stats"]["flag_count"][0] == 0
+    assert lit["stats"]["flag_count"][1] == 0  # never overcommits
