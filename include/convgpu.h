@@ -52,6 +52,13 @@ typedef enum {
   CONVGPU_RANDOM_FIT = 3   /* uniform among paused ("Random"), Philox-keyed */
 } convgpu_policy_t;
 
+/* OR-ed into the policy argument of convgpu_replay: replay under the literal
+ * re-select-on-every-release reading (R1-LIT, SURVEY §8(f)
+ * NEXT-1) instead of R1's sticky fill target.  Partial holds are kept, so
+ * deadlocks can occur and are reported by CONVGPU_FLAG_DEADLOCK.  Runs on the
+ * warp-per-trace kernel (AUTO selects it; LANE_PER_TRACE is -EINVAL). */
+#define CONVGPU_DISPATCH_LITERAL 0x100
+
 /* Op kinds: op_arg = kind << 30 | size_mib (size < 2^30).  The replay maps
  * the wrapper-module API classes of Table II: allocation APIs ->
  * ALLOC, cudaFree -> FREE, __cudaUnregisterFatBinary /
@@ -145,7 +152,8 @@ typedef struct {
  * P:149.  One warp per trace; the event loop, policy selection, outputs,
  * digests and the statistics reduction all run in the kernel.
  * capacity_mib: GPU memory to share, 1 .. CONVGPU_CAPACITY_LIMIT-1.
- * policy: convgpu_policy_t.  n may be 0 (no-op).
+ * policy: convgpu_policy_t, optionally | CONVGPU_DISPATCH_LITERAL.  n may be 0
+ * (no-op).
  * Errors: -EINVAL for NULL traces/out/arrays, n_containers or n_ops out of
  * range, policy out of range, capacity out of range, overhead out of range,
  * kernel_variant > 2, host pointers, range_digest without range_size; -ENODEV;

@@ -23,6 +23,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 SO_PATH = os.path.join(_PKG, "libconvgpu.so")
 
 FIFO, BEST_FIT, RECENT_FIT, RANDOM_FIT = 0, 1, 2, 3
+LITERAL = 0x100  # CONVGPU_DISPATCH_LITERAL: OR into a policy for the R1-LIT reading
 POLICY = {"fifo": FIFO, "best_fit": BEST_FIT, "recent_fit": RECENT_FIT, "random_fit": RANDOM_FIT}
 ALLOC, FREE, FINISH, NOP = 0, 1, 2, 3
 NONE32, NONE8 = 0xFFFFFFFF, 0xFF
@@ -107,7 +108,14 @@ def _check(rc: int, what: str):
 
 
 def _pol(policy) -> int:
-    return POLICY[policy] if isinstance(policy, str) else int(policy)
+    """'fifo' | 'best_fit' | 'recent_fit' | 'random_fit', optionally with a
+    '+literal' suffix, or the integer convgpu_policy_t [| LITERAL]."""
+    if isinstance(policy, str):
+        base, _, mode = policy.partition("+")
+        if mode not in ("", "literal"):
+            raise ConvgpuError(f"unknown dispatch reading {mode!r}")
+        return POLICY[base] | (LITERAL if mode else 0)
+    return int(policy)
 
 
 def _ptr(t) -> Optional[int]:

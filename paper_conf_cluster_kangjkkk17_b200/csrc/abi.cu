@@ -51,7 +51,10 @@ int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
   if (!t) return -EINVAL;
   if (t->n_containers < 1 || t->n_containers > CONVGPU_MAX_CONTAINERS) return -EINVAL;
   if (t->n_ops < 1 || t->n_ops > CONVGPU_MAX_OPS) return -EINVAL;
-  if (policy < 0 || policy > 3) return -EINVAL;
+  if (policy < 0 || (policy & ~(0xFF | CONVGPU_DISPATCH_LITERAL)) || (policy & 0xFF) > 3)
+    return -EINVAL;
+  if ((policy & CONVGPU_DISPATCH_LITERAL) && t->kernel_variant == CONVGPU_KERNEL_LANE_PER_TRACE)
+    return -EINVAL;
   if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
   if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
   if (t->kernel_variant > CONVGPU_KERNEL_LANE_PER_TRACE) return -EINVAL;
@@ -91,6 +94,7 @@ uint32_t auto_variant(uint64_t count, int policy) {
 }
 
 cudaError_t launch_any(const convgpu::ReplayArgs& a, int policy, uint32_t variant, cudaStream_t s) {
+  if (policy & CONVGPU_DISPATCH_LITERAL) variant = CONVGPU_KERNEL_WARP_PER_TRACE;
   if (variant == CONVGPU_KERNEL_AUTO) variant = auto_variant(a.count, policy);
   if (variant == CONVGPU_KERNEL_LANE_PER_TRACE) return convgpu::launch_replay_lpt(a, policy, s);
   return convgpu::launch_replay(a, policy, use_bulk(a), s);

@@ -57,11 +57,13 @@ static_assert(sizeof(WarpStats) == 96, "WarpStats layout");
 // cx.wait: d_1 before arrival, then the suspended-time accumulator.
 // cx.adm: admission (tick << 6 | rank); suspension number while paused.
 constexpr uint32_t kHeaderBytes = 128;
-constexpr uint32_t kCsBytes = 64 * 16, kCxBytes = 64 * 8;
+// ca[64]: explicit assignment a per container, used only by the literal
+// reading R1-LIT (partial holds are kept, so a is not derivable).
+constexpr uint32_t kCsBytes = 64 * 16, kCxBytes = 64 * 8, kCaBytes = 64 * 4;
 
 __host__ __device__ inline uint32_t in_words(uint32_t n, uint32_t K) { return (2 + 2 * K) * n; }
 __host__ __device__ inline uint32_t warp_region_bytes(uint32_t n, uint32_t K) {
-  uint32_t b = kHeaderBytes + kCsBytes + kCxBytes + 2 * in_words(n, K) * 4;
+  uint32_t b = kHeaderBytes + kCsBytes + kCxBytes + kCaBytes + 2 * in_words(n, K) * 4;
   return (b + 15u) & ~15u;
 }
 
@@ -107,7 +109,8 @@ __device__ __forceinline__ uint32_t redux_max(uint32_t v) {
 
 // ---------------------------------------------------------------- kernel
 // NF: compile-time container count (64) or 0 = runtime p.n.
-template <int POLICY, bool BULK, int NF>
+// LIT: the literal re-select-on-every-release reading R1-LIT (NEXT-1).
+template <int POLICY, bool BULK, int NF, bool LIT>
 __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) unsigned char smem[];
   const uint32_t lane = threadIdx.x & 31u, lane32 = lane + 32u;
@@ -121,7 +124,8 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
   unsigned long long* racc = reinterpret_cast<unsigned long long*>(base + 112);  // [cur, acc]
   uint4* cs = reinterpret_cast<uint4*>(base + kHeaderBytes);
   uint2* cx = reinterpret_cast<uint2*>(base + kHeaderBytes + kCsBytes);
-  uint32_t* inbuf = reinterpret_cast<uint32_t*>(base + kHeaderBytes + kCsBytes + kCxBytes);
+  uint32_t* ca = reinterpret_cast<uint32_t*>(base + kHeaderBytes + kCsBytes + kCxBytes);
+  uint32_t* inbuf = reinterpret_cast<uint32_t*>(base + kHeaderBytes + kCsBytes + kCxBytes + kCaBytes);
 
   const uint64_t warps_per_block = blockDim.x >> 5;
   const uint64_t gw = (uint64_t)blockIdx.x * warps_per_block + wib;
@@ -205,6 +209,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
         }
         cs[c] = make_uint4(kNotArrived, R[c], D[c], L);
         cx[c] = make_uint2(K > 1 ? D[n + c] : 0u, kKeyNone);
+        if (LIT) ca[c] = 0;
         const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
         if (s == 0) key0 = key; else key1 = key;
       }
@@ -239,15 +244,16 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
         bool disp = false;
         if ((ust & kNotArrived) == kNotArrived) {
           // ARRIVE (Fig. 3b/3c; R2)
-          const uint32_t g = (target == kTargetNone) ? min(L, free_mem) : 0u;
+          const uint32_t g = (LIT || target == kTargetNone) ? min(L, free_mem) : 0u;
           free_mem -= g;
           peak_res = max(peak_res, cap - free_mem);
           if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
           uint32_t adm = kKeyNone;
           ust = 0;
+          if (LIT) ca[c] = g;
           if (g == L) {
             adm = (t << 6) | rank; ++rank; ust = kAdmitted;
-          } else if (g > 0) {
+          } else if (g > 0 && !LIT) {
             target = c; a_tg = g;
           }
           const uint32_t d1 = cx[c].x;
@@ -260,7 +266,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
           bool adv = true;
           if (kind == CONVGPU_OP_ALLOC) {
             const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
-            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
+            const uint32_t a = LIT ? ca[c] : ((ust & kAdmitted) ? L : (c == target ? a_tg : 0u));
             if (need > L) {
               ++n_rej;  // R10
             } else if (need <= a) {
@@ -275,7 +281,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
               ++seq;
               if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
               adv = false;
-              disp = (target == kTargetNone);
+              disp = LIT || (target == kTargetNone);
               cs[c].x = ust;
             }
           } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
@@ -283,7 +289,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             ust -= r;
             used_total -= r;
           } else if (kind == CONVGPU_OP_FINISH) {  // P:110, R18
-            const uint32_t a = (ust & kAdmitted) ? L : (c == target ? a_tg : 0u);
+            const uint32_t a = LIT ? ca[c] : ((ust & kAdmitted) ? L : (c == target ? a_tg : 0u));
             free_mem += a;
             used_total -= used;
             --live;
@@ -305,7 +311,77 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
         key1 = (c == lane32) ? nk : key1;
 
         // ---- DISPATCH (Fig. 3d; R1, R9) ----
-        if (disp) {
+        // ---- SELECT among paused ----
+        auto select_paused = [&]() -> uint32_t {
+          uint32_t sel;
+          if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
+            sel = pm_lo ? (uint32_t)(__ffs(pm_lo) - 1) : 32u + (uint32_t)(__ffs(pm_hi) - 1);
+          } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - a (a = 0 when selectable under R1)
+            uint32_t vf = 0, vm = kKeyNone;
+            if ((pm_lo >> lane) & 1u) {
+              const uint32_t need = Lm[lane] - (LIT ? ca[lane] : 0u);
+              if (need <= free_mem) vf = (need << 6) | (63u - lane);
+              vm = (need << 6) | lane;
+            }
+            if (lane32 < n && ((pm_hi >> lane) & 1u)) {
+              const uint32_t need = Lm[lane32] - (LIT ? ca[lane32] : 0u);
+              if (need <= free_mem) vf = max(vf, (need << 6) | (63u - lane32));
+              vm = min(vm, (need << 6) | lane32);
+            }
+            const uint32_t kf = redux_max(vf);
+            sel = kf ? 63u - (kf & 63u) : (redux_min(vm) & 63u);
+          } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
+            uint32_t v = 0;
+            if ((pm_lo >> lane) & 1u) v = ((cx[lane].y + 1u) << 6) | lane;
+            if (lane32 < n && ((pm_hi >> lane) & 1u)) v = max(v, ((cx[lane32].y + 1u) << 6) | lane32);
+            sel = redux_max(v) & 63u;
+          } else {  // RANDOM_FIT (R6)
+            const uint32_t clo = __popc(pm_lo);
+            const uint32_t m = clo + __popc(pm_hi);
+            const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                       (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+            ++draws;
+            const uint32_t jj = __umulhi(x.x, m);
+            sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+          }
+          return sel;
+        };
+        if (disp && LIT) {
+          // R1-LIT: while memory is free and someone is paused, the policy's
+          // pick receives min(free, L - a); partial holds are kept.
+          while (free_mem != 0 && (pm_lo | pm_hi) != 0u) {
+            const uint32_t x = select_paused();
+            ++n_sel;
+            uint4 st = cs[x];
+            const uint32_t Lx = st.w;
+            const uint32_t g = min(free_mem, Lx - ca[x]);
+            const uint32_t ax = ca[x] + g;
+            ca[x] = ax;
+            free_mem -= g;
+            peak_res = max(peak_res, cap - free_mem);
+            uint32_t ut = st.x;
+            if (ut & kPaused) {
+              const uint32_t pend = (st.y & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
+              const uint32_t uu = ut & kUsedMask;
+              if (uu + pend <= ax) {  // RESUME (R9)
+                used_total += pend;
+                peak_used = max(peak_used, used_total);
+                cx[x] = make_uint2(cx[x].x + t, kKeyNone);
+                if (x < 32) pm_lo &= ~(1u << x); else pm_hi &= ~(1u << (x - 32));
+                const uint32_t k = ((ut >> kKShift) & 7u) + 1u;
+                ut = (ut & ~(kUsedMask | kKMask | kPaused)) | (uu + pend) | kFirst | (k << kKShift);
+                const uint32_t nkx = ((t + st.z) << 6) | x;
+                key0 = (x == lane) ? nkx : key0;
+                key1 = (x == lane32) ? nkx : key1;
+                st.y = R[k * n + x];
+                st.z = (k + 1 < K) ? D[(k + 1) * n + x] : 0u;
+              }
+            }
+            if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+            if (ax == Lx) { cx[x].y = (t << 6) | rank; ++rank; ut |= kAdmitted; }
+            cs[x] = make_uint4(ut, st.y, st.z, Lx);
+          }
+        } else if (disp) {
           for (;;) {
             if (target != kTargetNone) {
               const uint32_t tg = target;
@@ -346,38 +422,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
               break;
             }
             if ((pm_lo | pm_hi) == 0u) break;
-            // ---- SELECT among paused ----
-            uint32_t sel;
-            if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
-              sel = pm_lo ? (uint32_t)(__ffs(pm_lo) - 1) : 32u + (uint32_t)(__ffs(pm_hi) - 1);
-            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
-              uint32_t vf = 0, vm = kKeyNone;
-              if ((pm_lo >> lane) & 1u) {
-                const uint32_t need = Lm[lane];
-                if (need <= free_mem) vf = (need << 6) | (63u - lane);
-                vm = (need << 6) | lane;
-              }
-              if (lane32 < n && ((pm_hi >> lane) & 1u)) {
-                const uint32_t need = Lm[lane32];
-                if (need <= free_mem) vf = max(vf, (need << 6) | (63u - lane32));
-                vm = min(vm, (need << 6) | lane32);
-              }
-              const uint32_t kf = redux_max(vf);
-              sel = kf ? 63u - (kf & 63u) : (redux_min(vm) & 63u);
-            } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
-              uint32_t v = 0;
-              if ((pm_lo >> lane) & 1u) v = ((cx[lane].y + 1u) << 6) | lane;
-              if (lane32 < n && ((pm_hi >> lane) & 1u)) v = max(v, ((cx[lane32].y + 1u) << 6) | lane32);
-              sel = redux_max(v) & 63u;
-            } else {  // RANDOM_FIT (R6)
-              const uint32_t clo = __popc(pm_lo);
-              const uint32_t m = clo + __popc(pm_hi);
-              const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
-                                         (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
-              ++draws;
-              const uint32_t jj = __umulhi(x.x, m);
-              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
-            }
+            const uint32_t sel = select_paused();
             target = sel;
             a_tg = 0;
             ++n_sel;
@@ -486,11 +531,11 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
 }
 
 // ---------------------------------------------------------------- launcher
-template <int POLICY, bool BULK, int NF>
+template <int POLICY, bool BULK, int NF, bool LIT>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
   const uint32_t warps = kReplayThreads / 32;
   const size_t smem = (size_t)warps * warp_region_bytes(a.n, a.K);
-  auto kern = replay_kernel<POLICY, BULK, NF>;
+  auto kern = replay_kernel<POLICY, BULK, NF, LIT>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0, per_sm = 0;
@@ -510,19 +555,22 @@ static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
 }
 
 template <int POLICY>
-static cudaError_t launch_p(const ReplayArgs& a, bool bulk, cudaStream_t stream) {
-  if (a.n == 64) return bulk ? launch_t<POLICY, true, 64>(a, stream) : launch_t<POLICY, false, 64>(a, stream);
-  return bulk ? launch_t<POLICY, true, 0>(a, stream) : launch_t<POLICY, false, 0>(a, stream);
+static cudaError_t launch_p(const ReplayArgs& a, bool bulk, bool lit, cudaStream_t stream) {
+  if (lit) return bulk ? launch_t<POLICY, true, 0, true>(a, stream) : launch_t<POLICY, false, 0, true>(a, stream);
+  if (a.n == 64)
+    return bulk ? launch_t<POLICY, true, 64, false>(a, stream) : launch_t<POLICY, false, 64, false>(a, stream);
+  return bulk ? launch_t<POLICY, true, 0, false>(a, stream) : launch_t<POLICY, false, 0, false>(a, stream);
 }
 
 }  // namespace wpt
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream) {
-  switch (policy) {
-    case CONVGPU_FIFO: return wpt::launch_p<CONVGPU_FIFO>(a, bulk, stream);
-    case CONVGPU_BEST_FIT: return wpt::launch_p<CONVGPU_BEST_FIT>(a, bulk, stream);
-    case CONVGPU_RECENT_FIT: return wpt::launch_p<CONVGPU_RECENT_FIT>(a, bulk, stream);
-    case CONVGPU_RANDOM_FIT: return wpt::launch_p<CONVGPU_RANDOM_FIT>(a, bulk, stream);
+  const bool lit = (policy & CONVGPU_DISPATCH_LITERAL) != 0;
+  switch (policy & 0xFF) {
+    case CONVGPU_FIFO: return wpt::launch_p<CONVGPU_FIFO>(a, bulk, lit, stream);
+    case CONVGPU_BEST_FIT: return wpt::launch_p<CONVGPU_BEST_FIT>(a, bulk, lit, stream);
+    case CONVGPU_RECENT_FIT: return wpt::launch_p<CONVGPU_RECENT_FIT>(a, bulk, lit, stream);
+    case CONVGPU_RANDOM_FIT: return wpt::launch_p<CONVGPU_RANDOM_FIT>(a, bulk, lit, stream);
   }
   return cudaErrorInvalidValue;
 }

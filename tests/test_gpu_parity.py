@@ -277,3 +277,35 @@ def test_stats_accumulate_across_calls_and_streams(cg, orc):
     st = cg.stats_dict(out.stats_np())
     assert st["traces"] == 2 * ref["traces"] and st["events"] == 2 * ref["events"]
     assert st["max_makespan"] == ref["max_makespan"]
+
+
+# ---------------------------------------------------------------- NEXT-1
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("case", [(4, 3, 8, 0, "valid", 2000), (7, 5, 16, 2, "mixed", 1500),
+                                  (64, 4, 512, 66, "valid", 400)], ids=["n4", "n7mixed", "n64"])
+def test_literal_reading_parity(cg, orc, policy, case):
+    """R1-LIT (literal re-select-on-every-release) on the GPU vs the oracle,
+    including the traces it deadlocks (flag bit 0, zeroed outputs)."""
+    n, K, cap, ovh, mode, count = case
+    b = W.random_batch(77 + n, count, n, K, cap, ovh=ovh, mode=mode, max_arrival_step=1,
+                       limit_choices=range(1, cap + 1))
+    pid = POLS.index(policy) | 0x100
+    ref = orc.replay_batch(b, cap, pid, tid_base=9, rand_seed=4, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=9)
+    out = _gpu_replay(cg, tr, cap, policy + "+literal", seed=4, ovh=ovh)
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_literal_reading_deadlocks_on_paper_mimic(cg, orc, policy):
+    """The paper-mimic workload under R1-LIT vs R1 on the GPU:
+    the literal reading deadlocks a share of traces, R1 none (P:7)."""
+    w = W.CONFIGS["mimic"]
+    N = 2000
+    tr = cg.generate(w.gen, 0, N)
+    lit = _gpu_replay(cg, tr, w.cap, policy + "+literal", seed=w.rand_seed, ovh=w.ovh)
+    ref = orc.replay_range(w, POLS.index(policy) | 0x100, 0, N, full=True)
+    _compare(cg, lit, ref)
+    sticky = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, ovh=w.ovh, full=False)
+    assert cg.stats_dict(sticky.stats_np())["flag_count"][0] == 0
