@@ -57,9 +57,10 @@ enum { W_KEY = 0, W_L = 1, W_UST = 2, W_ADM = 3, W_CW = 4, W_ND = 5, W_BASE_WORD
 //        the suspension number while paused (Recent-Fit scan fallback).
 // W_ND:  delta to add at the container's next scheduling (d_0 before
 //        arrival, then d_{k+1}); the finish tick after FINISH.
-// Best-Fit adds W_RK (byte0 rank_of[j], byte1 gs[j], byte2 pi[j]) and W_LS
-// (limits sorted by (L, index)); Recent-Fit adds a kStack-byte stack.
-__host__ __device__ constexpr int extra_words(int policy) { return policy == CONVGPU_BEST_FIT ? 2 : 0; }
+// Best-Fit adds W_RK (byte0 rank_of[j], byte1 gs[j], byte2 pi[j]: rank of
+// container j in (L, index) order, first rank of rank j's limit, container
+// of rank j); Recent-Fit adds a kStack-byte stack.
+__host__ __device__ constexpr int extra_words(int policy) { return policy == CONVGPU_BEST_FIT ? 1 : 0; }
 
 __host__ __device__ inline size_t warp_bytes(int policy, uint32_t n) {
   size_t b = (size_t)(W_BASE_WORDS + extra_words(policy)) * n * 32 * 4;
@@ -112,7 +113,6 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   uint32_t* const s_cw = S + (size_t)W_CW * n * 32;
   uint32_t* const s_nd = S + (size_t)W_ND * n * 32;
   uint32_t* const s_rk = S + (size_t)(W_BASE_WORDS + 0) * n * 32;  // Best-Fit only
-  uint32_t* const s_ls = S + (size_t)(W_BASE_WORDS + 1) * n * 32;  // Best-Fit only
   uint8_t* const s_stk = reinterpret_cast<uint8_t*>(W0 + (size_t)W_BASE_WORDS * n * 32) + lane * 4;
 #define AT(arr, c) (arr)[(c) * 32u]
 #define RKB(j, b) reinterpret_cast<uint8_t*>(&AT(s_rk, (j)))[b]
@@ -213,7 +213,6 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           RKB(c, 0) = (uint8_t)r;
           RKB(r, 1) = (uint8_t)gsr;
           RKB(r, 2) = (uint8_t)c;
-          AT(s_ls, r) = Lc;
         }
       } else {
         for (uint32_t c = 0; c < n; ++c) {
@@ -228,7 +227,6 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           RKB(c, 0) = (uint8_t)r;
           RKB(r, 1) = (uint8_t)lt;
           RKB(r, 2) = (uint8_t)c;
-          AT(s_ls, r) = Lc;
         }
       }
     }
@@ -408,7 +406,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             for (int it = 0; it < 7; ++it) {
               if (lo < hi) {
                 const uint32_t mid = (lo + hi) >> 1;
-                if (AT(s_ls, mid) <= free_mem) lo = mid + 1; else hi = mid;
+                if (AT(s_L, RKB(mid, 2)) <= free_mem) lo = mid + 1; else hi = mid;
               }
             }
             uint32_t ml, mh;
@@ -545,9 +543,8 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
 
 template <int POLICY, int NF, int KF>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
-  // Best-Fit's rank tables make a warp's slice 64 KB: one warp per CTA packs
-  // three per SM; the others fit two 2-warp CTAs (four warps) per SM.
-  const int threads = POLICY == CONVGPU_BEST_FIT ? 32 : kLptThreads;
+  // two 2-warp CTAs (four warps) per SM for every policy
+  const int threads = kLptThreads;
   const size_t smem = (size_t)(threads / 32) * warp_bytes(POLICY, a.n);
   auto kern = replay_lpt_kernel<POLICY, NF, KF>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
