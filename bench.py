@@ -180,17 +180,18 @@ def cpu_baseline(w, sample):
                       f"(ids 0..{sample - 1}), single-threaded C oracle, {dt:.1f} s"}
 
 
-def traffic_from_profiles(workload, traces):
-    """dram bytes per replay launch from the committed ncu --set full summary."""
+def ncu_summary(workload, traces):
+    """DRAM bytes per replay launch and the limiter evidence from the committed
+    ncu --set full summary (profiles/ncu_full_summary.json), if it matches."""
     p = os.path.join(ROOT, "profiles", "ncu_full_summary.json")
     try:
         with open(p) as f:
             d = json.load(f)
         if d.get("workload") == workload and int(d.get("traces")) == traces:
-            return d.get("dram_bytes_per_launch")
+            return d
     except Exception:
         pass
-    return None
+    return {}
 
 
 def run_ours(args, rank, local_rank, world):
@@ -295,14 +296,18 @@ def run_ours(args, rank, local_rank, world):
     avg_launch_s = statistics.mean(launch_ms.values()) / 1e3
     peak, peak_src = measured_peak()
     achieved = bytes_per_launch / avg_launch_s / 1e9
+    ncu = ncu_summary(w.name, Nr)
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic_from_profiles(w.name, Nr),
+                "frac": achieved / peak, "traffic": ncu.get("dram_bytes_per_launch"),
+                "ncu_limiter": ncu.get("limiter"), "ncu_source": ncu.get("source"),
                 "kernel": "replay kernels: " + ", ".join(
                     f"{p}={kernel_of(p)}" for p in POLICIES),
                 "algorithmic_bytes_per_launch": bytes_per_launch,
                 "bytes_per_event": (in_b + out_b) / per_trace_events, "peak_source": peak_src,
                 "avg_launch_ms": avg_launch_s * 1e3,
-                "note": "issue/latency-bound warp-serial event loop; see DESIGN.md §Roofline"}
+                "note": "HBM is the roofline bound (a few integer ops per byte); the achieved "
+                        "rate is limited by each trace's serial event chain (latency / issue), "
+                        "see ncu_limiter and DESIGN.md §6.4"}
 
     result = None
     if rank == 0:

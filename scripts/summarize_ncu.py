@@ -72,7 +72,12 @@ def full(rep, tag, events_per_launch, traffic, workload, traces):
         with open(os.path.join(PROF, "ncu_full_summary.json"), "w") as f:
             json.dump({"workload": workload, "traces": traces, "source": f"{tag}_ncu_full.json",
                        "dram_bytes_per_launch": statistics.mean(per),
-                       "per_kernel": {k["kernel"]: k["dram_bytes_per_launch"] for k in kernels}},
+                       "per_kernel": {k["kernel"]: k["dram_bytes_per_launch"] for k in kernels},
+                       "limiter": {k["kernel"]: {
+                           "warp_instructions_per_event": round(k.get("warp_instructions_per_event", 0), 2),
+                           "issue_active_pct": float(k["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"]),
+                           "active_lanes": float(k["smsp__thread_inst_executed_per_inst_executed.ratio"]["value"]),
+                           "top_stalls": k["stall_share_top"]} for k in kernels}},
                       f, indent=1)
 
 
