@@ -201,10 +201,18 @@ def run_ours(args, rank, local_rank, world):
     import paper_conf_cluster_kangjkkk17_b200 as cg
     from paper_conf_cluster_kangjkkk17_b200 import dist as cgd
 
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+    # one process per GPU; ranks beyond the visible devices share them (only
+    # useful with CONVGPU_DIST_BACKEND=gloo, to exercise the N>1 flow on a
+    # one-GPU box — NCCL needs one rank per device)
+    ndev = torch.cuda.device_count()
+    dev = torch.device("cuda", local_rank % ndev)
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("CONVGPU_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     cg.lib()
     w = W.CONFIGS[args.workload]
     Nr = args.traces or (w.n_traces if args.workload != "c3" else w.n_traces // world)
@@ -250,7 +258,7 @@ def run_ours(args, rank, local_rank, world):
     sampler = None
     if not args.profile:
         vis = os.environ.get("CUDA_VISIBLE_DEVICES")
-        phys = int(vis.split(",")[local_rank]) if vis else local_rank
+        phys = int(vis.split(",")[dev.index]) if vis else dev.index
         sampler = ClockSampler(phys)
         sampler.start()
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
