@@ -114,3 +114,11 @@ def test_product_package_does_not_import_oracle():
                 txt = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "oracle.h" not in txt and "liboracle" not in txt, f
+
+
+def test_missing_extension_fails_loudly(monkeypatch, tmp_path):
+    """No CPU fallback: without libconvgpu.so every call raises."""
+    monkeypatch.setattr(cg, "SO_PATH", str(tmp_path / "missing.so"))
+    monkeypatch.setattr(cg, "_lib", None)
+    with pytest.raises(cg.ConvgpuError):
+        cg.lib()

@@ -309,3 +309,49 @@ def test_literal_reading_deadlocks_on_paper_mimic(cg, orc, policy):
     _compare(cg, lit, ref)
     sticky = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, ovh=w.ovh, full=False)
     assert cg.stats_dict(sticky.stats_np())["flag_count"][0] == 0
+
+
+def _extreme_batch(seed, count, n, K):
+    """Values at the ABI limits: capacity 2^26-1, limits up to it, ALLOC sizes
+    up to 2^30-1 (over-limit ones are rejected), large deltas with trace
+    horizons at exactly 2^26-1 (valid) and >= 2^26 (TICK_RANGE)."""
+    rng = np.random.default_rng(seed)
+    cap = (1 << 26) - 1
+    parts = [W.random_batch(seed + j, count // 3, n, K, 16, ovh=1, mode=m, max_arrival_step=2,
+                            limit_choices=range(1, 17))
+             for j, m in enumerate(("valid", "over", "delayed"))]
+    cat = lambda f: np.concatenate([getattr(b, f) for b in parts])  # noqa: E731
+    arrival, limit, delta, arg = cat("arrival"), cat("limit"), cat("delta"), cat("arg")
+    N = arrival.shape[0]
+    scale = cap // 16
+    limit = np.minimum(limit.astype(np.uint64) * scale, cap).astype(np.uint32)
+    kinds = arg >> 30
+    sizes = (arg & 0x3FFFFFFF).astype(np.uint64) * scale
+    big = (rng.random(sizes.shape) < 0.05) & (kinds == 0)  # huge ALLOCs: rejected
+    sizes = np.where(big, (1 << 30) - 1, np.minimum(sizes, (1 << 30) - 1)).astype(np.uint32)
+    arg = ((kinds << 30) | sizes).astype(np.uint32)
+    unit = (1 << 26) // (4 * (n * K + 1))
+    delta = (delta.astype(np.uint64) * unit).astype(np.uint32)
+    arrival = (arrival.astype(np.uint64) * unit).astype(np.uint32)
+    for i in range(N):  # horizon = max arrival + sum of deltas
+        h = int(arrival[i].max()) + int(delta[i].astype(np.uint64).sum())
+        if i % 5 == 0:
+            delta[i, K - 1, 0] += np.uint32((1 << 26) - 1 - h)  # exactly representable
+        elif i % 5 == 1:
+            delta[i, K - 1, 0] += np.uint32((1 << 26) - h)      # one past: TICK_RANGE
+    return W.Batch(n, K, arrival, limit, delta, arg), cap, scale  # overhead = 1 unit
+
+
+@pytest.mark.parametrize("kernel", KERNELS)
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("nk", [(8, 4), (64, 8)], ids=["n8K4", "n64K8"])
+def test_extreme_values(cg, orc, kernel, policy, nk):
+    n, K = nk
+    b, cap, ovh = _extreme_batch(31 + n, 300, n, K)
+    ref = orc.replay_batch(b, cap, policy, tid_base=2**63 + 5, rand_seed=2**64 - 1, ovh=ovh)
+    st = ref["stats"]
+    assert st["flag_count"][5] > 0 and st["n_select"] > 0 and st["n_rejected"] > 0
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=2**63 + 5)
+    out = _gpu_replay(cg, tr, cap, policy, seed=2**64 - 1, ovh=ovh, kernel=kernel)
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
