@@ -93,7 +93,9 @@ uint32_t auto_variant(uint64_t count, int policy) {
   return big ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
 }
 
-cudaError_t launch_any(const convgpu::ReplayArgs& a, int policy, uint32_t variant, cudaStream_t s) {
+cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cudaStream_t s) {
+  a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.wait) &&
+                aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
   if (policy & CONVGPU_DISPATCH_LITERAL) variant = CONVGPU_KERNEL_WARP_PER_TRACE;
   if (variant == CONVGPU_KERNEL_AUTO) variant = auto_variant(a.count, policy);
   if (variant == CONVGPU_KERNEL_LANE_PER_TRACE) return convgpu::launch_replay_lpt(a, policy, s);

@@ -25,6 +25,7 @@ struct ReplayArgs {
   uint64_t* range_digest;
   uint64_t range_size;
   uint64_t grid_override;  // 0 = occupancy-sized persistent grid
+  uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
 };
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream);

@@ -98,6 +98,10 @@ __device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi
 }
 
 // NF, KF: compile-time container / op counts (64, 4 for the configs) or 0.
+__device__ __forceinline__ uint32_t comp(const uint4& v, int j) {
+  return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
+}
+
 template <int POLICY, int NF, int KF>
 __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
@@ -154,31 +158,67 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     uint32_t bad = 0, lsum = 0, amax = 0, prev = 0;
 #pragma unroll
     for (int j = 0; j < 8; ++j) gmin[j] = kKeyNone;
-    for (uint32_t c = 0; c < n; ++c) {
-      const uint32_t a = __ldg(A + c), L = __ldg(Lg + c);
-      if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
-      if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
-      prev = a;
-      amax = max(amax, a);
-      uint32_t d0 = 0, d1 = 0, w0 = 0;
-      for (uint32_t k = 0; k < K; ++k) {
-        const uint32_t d = __ldg(trace_delta + (size_t)k * n + c);
-        const uint32_t w = __ldg(trace_arg + (size_t)k * n + c);
-        lsum = min(lsum + min(d, kTickLimit), kTickLimit);
-        if (((w >> 30) == CONVGPU_OP_FINISH) != (k + 1 == K)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
-        if (k == 0) { d0 = d; w0 = w; }
-        if (k == 1) d1 = d;
-      }
-      const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
-      AT(s_key, c) = key;
-      AT(s_L, c) = L;
-      AT(s_ust, c) = kNotArrived;
-      AT(s_adm, c) = d1;
-      AT(s_cw, c) = w0;
-      AT(s_nd, c) = d0;
-      const uint32_t g = c >> 3;
+    if (NF == 64 && KF == 4 && p.aligned16) {
+      // 16-byte loads, 4 containers per step, every load of a step in flight
+      const uint4* A4 = reinterpret_cast<const uint4*>(A);
+      const uint4* L4 = reinterpret_cast<const uint4*>(Lg);
+      const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
+      const uint4* R4 = reinterpret_cast<const uint4*>(trace_arg);
 #pragma unroll
-      for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? min(gmin[j], key) : gmin[j];
+      for (uint32_t q = 0; q < 16; ++q) {
+        const uint4 a4 = __ldg(A4 + q), l4 = __ldg(L4 + q);
+        uint4 d4[4], w4[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) { d4[k] = __ldg(D4 + k * 16 + q); w4[k] = __ldg(R4 + k * 16 + q); }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t c = 4 * q + j, a = comp(a4, j), L = comp(l4, j);
+          if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+          if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
+          prev = a;
+          amax = max(amax, a);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            lsum = min(lsum + min(comp(d4[k], j), kTickLimit), kTickLimit);
+            if (((comp(w4[k], j) >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+          }
+          const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
+          AT(s_key, c) = key;
+          AT(s_L, c) = L;
+          AT(s_ust, c) = kNotArrived;
+          AT(s_adm, c) = comp(d4[1], j);
+          AT(s_cw, c) = comp(w4[0], j);
+          AT(s_nd, c) = comp(d4[0], j);
+          gmin[c >> 3] = min(gmin[c >> 3], key);
+        }
+      }
+    } else {
+      for (uint32_t c = 0; c < n; ++c) {
+        const uint32_t a = __ldg(A + c), L = __ldg(Lg + c);
+        if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+        if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
+        prev = a;
+        amax = max(amax, a);
+        uint32_t d0 = 0, d1 = 0, w0 = 0;
+        for (uint32_t k = 0; k < K; ++k) {
+          const uint32_t d = __ldg(trace_delta + (size_t)k * n + c);
+          const uint32_t w = __ldg(trace_arg + (size_t)k * n + c);
+          lsum = min(lsum + min(d, kTickLimit), kTickLimit);
+          if (((w >> 30) == CONVGPU_OP_FINISH) != (k + 1 == K)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+          if (k == 0) { d0 = d; w0 = w; }
+          if (k == 1) d1 = d;
+        }
+        const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
+        AT(s_key, c) = key;
+        AT(s_L, c) = L;
+        AT(s_ust, c) = kNotArrived;
+        AT(s_adm, c) = d1;
+        AT(s_cw, c) = w0;
+        AT(s_nd, c) = d0;
+        const uint32_t g = c >> 3;
+  #pragma unroll
+        for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? min(gmin[j], key) : gmin[j];
+      }
     }
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     if (POLICY == CONVGPU_BEST_FIT) {
@@ -246,28 +286,69 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     uint64_t dig = 0, swait = 0;
     uint32_t mfin = 0;
     const uint64_t ob = ti * n;
-    for (uint32_t c = 0; c < n; ++c) {
-      uint32_t at = kKeyNone, ar = 0xFFu, wt = 0, fn = 0;
-      if (!stopped) {
-        const uint32_t u = AT(s_ust, c);
-        if (u & kAdmitted) {
-          const uint32_t adm = AT(s_adm, c);
-          at = adm >> 6;
-          ar = adm & 63u;
+    if (NF == 64 && KF == 4 && p.aligned16) {
+      const uint4* A4 = reinterpret_cast<const uint4*>(A);
+      const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
+#pragma unroll 4
+      for (uint32_t q = 0; q < 16; ++q) {
+        uint4 a4 = make_uint4(0, 0, 0, 0), d4[4];
+        if (!stopped) {
+          a4 = __ldg(A4 + q);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) d4[k] = __ldg(D4 + k * 16 + q);
         }
-        fn = AT(s_nd, c);
-        uint32_t sd = __ldg(A + c);  // R17: wait = finish - arrival - sum of deltas
-        for (uint32_t k = 0; k < K; ++k) sd += __ldg(trace_delta + (size_t)k * n + c);
-        wt = fn - sd;
+        uint32_t at[4], ar[4], wt[4], fn[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t c = 4 * q + j;
+          at[j] = kKeyNone; ar[j] = 0xFFu; wt[j] = 0; fn[j] = 0;
+          if (!stopped) {
+            const uint32_t u = AT(s_ust, c);
+            if (u & kAdmitted) {
+              const uint32_t adm = AT(s_adm, c);
+              at[j] = adm >> 6;
+              ar[j] = adm & 63u;
+            }
+            fn[j] = AT(s_nd, c);
+            // R17: wait = finish - arrival - sum of deltas
+            wt[j] = fn[j] - comp(a4, j) - comp(d4[0], j) - comp(d4[1], j) - comp(d4[2], j) -
+                    comp(d4[3], j);
+          }
+          const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
+          dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
+          mfin = max(mfin, fn[j]);
+          swait += wt[j];
+        }
+        if (p.admit_tick) reinterpret_cast<uint4*>(p.admit_tick + ob)[q] = make_uint4(at[0], at[1], at[2], at[3]);
+        if (p.admit_rank)
+          reinterpret_cast<uint32_t*>(p.admit_rank + ob)[q] = ar[0] | (ar[1] << 8) | (ar[2] << 16) | (ar[3] << 24);
+        if (p.wait) reinterpret_cast<uint4*>(p.wait + ob)[q] = make_uint4(wt[0], wt[1], wt[2], wt[3]);
+        if (p.finish) reinterpret_cast<uint4*>(p.finish + ob)[q] = make_uint4(fn[0], fn[1], fn[2], fn[3]);
       }
-      if (p.admit_tick) p.admit_tick[ob + c] = at;
-      if (p.admit_rank) p.admit_rank[ob + c] = (uint8_t)ar;
-      if (p.wait) p.wait[ob + c] = wt;
-      if (p.finish) p.finish[ob + c] = fn;
-      const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar << 48) ^ (uint64_t)at);
-      dig += mix64(h1 ^ (((uint64_t)wt << 32) | fn));
-      mfin = max(mfin, fn);
-      swait += wt;
+    } else {
+      for (uint32_t c = 0; c < n; ++c) {
+        uint32_t at = kKeyNone, ar = 0xFFu, wt = 0, fn = 0;
+        if (!stopped) {
+          const uint32_t u = AT(s_ust, c);
+          if (u & kAdmitted) {
+            const uint32_t adm = AT(s_adm, c);
+            at = adm >> 6;
+            ar = adm & 63u;
+          }
+          fn = AT(s_nd, c);
+          uint32_t sd = __ldg(A + c);  // R17: wait = finish - arrival - sum of deltas
+          for (uint32_t k = 0; k < K; ++k) sd += __ldg(trace_delta + (size_t)k * n + c);
+          wt = fn - sd;
+        }
+        if (p.admit_tick) p.admit_tick[ob + c] = at;
+        if (p.admit_rank) p.admit_rank[ob + c] = (uint8_t)ar;
+        if (p.wait) p.wait[ob + c] = wt;
+        if (p.finish) p.finish[ob + c] = fn;
+        const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar << 48) ^ (uint64_t)at);
+        dig += mix64(h1 ^ (((uint64_t)wt << 32) | fn));
+        mfin = max(mfin, fn);
+        swait += wt;
+      }
     }
     const uint32_t makespan = stopped ? 0u : mfin - __ldg(A);
     dig += mix64(((uint64_t)makespan << 32) | peak_res);
