@@ -78,11 +78,23 @@ __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_grou
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
-__device__ __forceinline__ bool bit64(uint32_t lo, uint32_t hi, uint32_t b) {
-  return ((b < 32 ? lo >> b : hi >> (b - 32)) & 1u) != 0;
+// PTX shifts clamp: a shift by >= 32 gives 0 (no guard instructions, unlike
+// C++ where it is undefined); b - 32 wraps to a huge count for b < 32.
+__device__ __forceinline__ uint32_t shl_c(uint32_t v, uint32_t s) {
+  uint32_t r;
+  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
+  return r;
 }
-__device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bool on) {
-  const uint32_t ml = (b < 32) ? (1u << b) : 0u, mh = (b >= 32 && b < 64) ? (1u << (b - 32)) : 0u;
+__device__ __forceinline__ uint32_t shr_c(uint32_t v, uint32_t s) {
+  uint32_t r;
+  asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
+  return r;
+}
+__device__ __forceinline__ bool bit64(uint32_t lo, uint32_t hi, uint32_t b) {  // b < 64
+  return ((shr_c(lo, b) | shr_c(hi, b - 32u)) & 1u) != 0;
+}
+__device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bool on) {  // b < 64
+  const uint32_t ml = shl_c(1u, b), mh = shl_c(1u, b - 32u);
   lo = on ? (lo | ml) : (lo & ~ml);
   hi = on ? (hi | mh) : (hi & ~mh);
 }
@@ -135,7 +147,8 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   uint32_t gmin[8];
   uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, seq = 0, rank = 0, draws = 0,
            n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
-  uint32_t pm_lo = 0, pm_hi = 0, pfc_lo = 0, pfc_hi = 0, pr_lo = 0, pr_hi = 0, sp = 0;
+  uint32_t pm_lo = 0, pm_hi = 0, pr_lo = 0, pr_hi = 0, sp = 0;
+  uint32_t pfc = kNoC;  // container whose op words were prefetched in the last iteration
   bool ru_scan = false;
   const uint32_t* trace_delta = nullptr;
   const uint32_t* trace_arg = nullptr;
@@ -143,9 +156,16 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   auto regroup = [&](uint32_t c) {  // re-min the group of container c
     const uint32_t g = c >> 3, b = g << 3;
     uint32_t m = kKeyNone;
+    if (NF != 0 && NF % 8 == 0) {  // whole groups: 8 loads in flight, min tree
+      uint32_t v[8];
 #pragma unroll
-    for (uint32_t j = 0; j < 8; ++j)
-      if (b + j < n) m = min(m, AT(s_key, b + j));
+      for (uint32_t j = 0; j < 8; ++j) v[j] = AT(s_key, b + j);
+      m = min(min(min(v[0], v[1]), min(v[2], v[3])), min(min(v[4], v[5]), min(v[6], v[7])));
+    } else {
+#pragma unroll
+      for (uint32_t j = 0; j < 8; ++j)
+        if (b + j < n) m = min(m, AT(s_key, b + j));
+    }
 #pragma unroll
     for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? m : gmin[j];
   };
@@ -273,7 +293,8 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     flags = bad;
     free_mem = cap; target = kNoC; a_tg = 0; used_total = 0; seq = 0; rank = 0; draws = 0;
     n_rej = 0; n_sel = 0; peak_res = 0; peak_used = 0; live = n; events = 0;
-    pm_lo = pm_hi = pfc_lo = pfc_hi = pr_lo = pr_hi = 0;
+    pm_lo = pm_hi = pr_lo = pr_hi = 0;
+    pfc = kNoC;
     sp = 0;
     ru_scan = false;
   };
@@ -388,8 +409,8 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   while (__any_sync(kFull, have)) {
     if (have && !tdone) {
       uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
-      const uint32_t pf_lo = pfc_lo, pf_hi = pfc_hi;  // previous iteration's group
-      pfc_lo = 0; pfc_hi = 0;
+      const uint32_t pf = pfc;  // previous iteration's group
+      pfc = kNoC;
       if (!dmode) {
         // ================= EVENT step (a2 + a3), branch-free =================
         const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
@@ -402,7 +423,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           const uint32_t t = kmin >> 6, c = kmin & 63u;
           cur_t = t;
           cp_wait1();  // every group but the previous iteration's is complete
-          if (bit64(pf_lo, pf_hi, c)) cp_wait0();
+          if (c == pf) cp_wait0();
           ++events;
           const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
           const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
@@ -572,9 +593,10 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
         AT(s_key, kc) = nkc;
         regroup(kc);
         if (pfk != 0xFFu) {  // op k word, delta of op k+1
-          if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + (size_t)pfk * n + kc);
-          if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + (size_t)(pfk + 1) * n + kc);
-          set64(pfc_lo, pfc_hi, kc, true);
+          const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
+          if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + off);
+          if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + off + n);
+          pfc = kc;
         }
       }
       cp_commit();
