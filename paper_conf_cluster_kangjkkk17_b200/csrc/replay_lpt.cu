@@ -407,201 +407,204 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
   // Lanes advance through their traces independently but start and finish
   // them together (warp vote below), so init/epilogue run converged.
   while (__any_sync(kFull, have)) {
-    if (have && !tdone) {
-      uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
-      const uint32_t pf = pfc;  // previous iteration's group
-      pfc = kNoC;
-      if (!dmode) {
-        // ================= EVENT step (a2 + a3), branch-free =================
-        const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
-        const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
-        const uint32_t kmin = min(min(m01, m23), min(m45, m67));
-        if (kmin == kKeyNone) {
-          if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
-          tdone = true;
-        } else {
-          const uint32_t t = kmin >> 6, c = kmin & 63u;
-          cur_t = t;
-          cp_wait1();  // every group but the previous iteration's is complete
-          if (c == pf) cp_wait0();
-          ++events;
-          const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
-          const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
-          const bool arr = (ust & kNotArrived) == kNotArrived;
-          const uint32_t kind = cw >> 30, r = cw & kSizeMask, used = ust & kUsedMask;
-          const bool isA = !arr && kind == CONVGPU_OP_ALLOC;
-          const bool isF = !arr && kind == CONVGPU_OP_FREE;
-          const bool isX = !arr && kind == CONVGPU_OP_FINISH;
-          const bool tnone = target == kNoC, ctg = c == target;
-          const uint32_t a_c = (ust & kAdmitted) ? L : (ctg ? a_tg : 0u);
-          // ARRIVE (Fig. 3b/3c; R2)
-          const uint32_t g = (arr && tnone) ? min(L, free_mem) : 0u;
-          const bool vadm = arr && g == L;
-          const bool vtgt = arr && !vadm && g > 0;
-          // ALLOC
-          const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
-          const bool rej = isA && need > L;                // R10
-          const bool grant = isA && !rej && need <= a_c;
-          const bool pause = isA && !rej && !grant;       // reply withheld
-          // FREE (R11)
-          const bool badfree = isF && r > used;
-          // ledger
-          free_mem = free_mem - g + (isX ? a_c : 0u);
-          used_total = used_total + (grant ? need - used : 0u) - ((isF && !badfree) ? r : 0u) -
-                       (isX ? used : 0u);
-          peak_res = max(peak_res, cap - free_mem);
-          peak_used = max(peak_used, used_total);
-          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
-          const bool clear_tg = isX && ctg;               // R20
-          target = vtgt ? c : (clear_tg ? kNoC : target);
-          a_tg = vtgt ? g : (clear_tg ? 0u : a_tg);
-          const uint32_t admv = (t << 6) | rank;
-          rank += vadm ? 1u : 0u;
-          n_rej += rej ? 1u : 0u;
-          live -= isX ? 1u : 0u;
-          if (pause) {
-            set64(pm_lo, pm_hi, c, true);
-            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(c, 0), true);
-            if (POLICY == CONVGPU_RECENT_FIT) {
-              if (sp < kStack) STK(sp) = (uint8_t)c;
-              ++sp;
-              ru_scan = ru_scan || sp > kStack;
-              AT(s_adm, c) = seq;  // suspension number (scan fallback)
-            }
-            ++seq;
-          }
-          // DISPATCH has work after a pause with no target (select) or a
-          // FINISH that leaves a target to fill or paused containers
-          dmode = (pause && tnone) || (isX && (target != kNoC || (pm_lo | pm_hi) != 0u));
-          if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true; }
-          const bool adv = !isX && !pause && !badfree;
-          // new state word
-          uint32_t nu = ust;
-          nu = grant ? ((ust & ~kUsedMask) | need | kFirst) : nu;
-          nu = (isF && !badfree) ? ust - r : nu;
-          nu = isX ? (ust & ~kUsedMask) : nu;
-          nu = pause ? (ust | kPaused) : nu;
-          nu = arr ? (vadm ? kAdmitted : 0u) : nu;
-          nu = (adv && !arr) ? nu + kKOne : nu;
-          AT(s_ust, c) = nu;
-          if (arr) AT(s_adm, c) = vadm ? admv : kKeyNone;
-          if (arr || isX) AT(s_nd, c) = arr ? am : t;     // d_1 / finish tick
-          kc = badfree ? kNoC : c;
-          nkc = adv ? (((t + nd) << 6) | c) : kKeyNone;
-          pfk = (adv && !arr) ? ((nu >> kKShift) & 7u) : 0xFFu;
-        }
-      } else {
-        // ====== one DISPATCH step at the triggering tick (R1, R9) ======
-        // A step = [SELECT if there is no fill target] + fill / resume / admit
-        // of the target; an admit keeps the lane in dispatch mode (the
-        // leftover cascades to the next selection, Fig. 3d).
-        const uint32_t t = cur_t;
-        if (target == kNoC) {
-          // ---- SELECT among paused; pm != 0 here ----
-          uint32_t sel;
-          if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
-            sel = ffs64(pm_lo, pm_hi);
-          } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
-            // R = #ranks with L <= free (limits sorted by (L, index))
-            uint32_t lo = 0, hi = n;
-#pragma unroll
-            for (int it = 0; it < 7; ++it) {
-              if (lo < hi) {
-                const uint32_t mid = (lo + hi) >> 1;
-                if (AT(s_L, RKB(mid, 2)) <= free_mem) lo = mid + 1; else hi = mid;
+    // inner loop: one micro-step per lane until every lane's trace is done
+    do {
+      if (have && !tdone) {
+        uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
+        const uint32_t pf = pfc;  // previous iteration's group
+        pfc = kNoC;
+        if (!dmode) {
+          // ================= EVENT step (a2 + a3), branch-free =================
+          const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
+          const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
+          const uint32_t kmin = min(min(m01, m23), min(m45, m67));
+          if (kmin == kKeyNone) {
+            if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
+            tdone = true;
+          } else {
+            const uint32_t t = kmin >> 6, c = kmin & 63u;
+            cur_t = t;
+            cp_wait1();  // every group but the previous iteration's is complete
+            if (c == pf) cp_wait0();
+            ++events;
+            const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
+            const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
+            const bool arr = (ust & kNotArrived) == kNotArrived;
+            const uint32_t kind = cw >> 30, r = cw & kSizeMask, used = ust & kUsedMask;
+            const bool isA = !arr && kind == CONVGPU_OP_ALLOC;
+            const bool isF = !arr && kind == CONVGPU_OP_FREE;
+            const bool isX = !arr && kind == CONVGPU_OP_FINISH;
+            const bool tnone = target == kNoC, ctg = c == target;
+            const uint32_t a_c = (ust & kAdmitted) ? L : (ctg ? a_tg : 0u);
+            // ARRIVE (Fig. 3b/3c; R2)
+            const uint32_t g = (arr && tnone) ? min(L, free_mem) : 0u;
+            const bool vadm = arr && g == L;
+            const bool vtgt = arr && !vadm && g > 0;
+            // ALLOC
+            const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
+            const bool rej = isA && need > L;                // R10
+            const bool grant = isA && !rej && need <= a_c;
+            const bool pause = isA && !rej && !grant;       // reply withheld
+            // FREE (R11)
+            const bool badfree = isF && r > used;
+            // ledger
+            free_mem = free_mem - g + (isX ? a_c : 0u);
+            used_total = used_total + (grant ? need - used : 0u) - ((isF && !badfree) ? r : 0u) -
+                         (isX ? used : 0u);
+            peak_res = max(peak_res, cap - free_mem);
+            peak_used = max(peak_used, used_total);
+            if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+            const bool clear_tg = isX && ctg;               // R20
+            target = vtgt ? c : (clear_tg ? kNoC : target);
+            a_tg = vtgt ? g : (clear_tg ? 0u : a_tg);
+            const uint32_t admv = (t << 6) | rank;
+            rank += vadm ? 1u : 0u;
+            n_rej += rej ? 1u : 0u;
+            live -= isX ? 1u : 0u;
+            if (pause) {
+              set64(pm_lo, pm_hi, c, true);
+              if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(c, 0), true);
+              if (POLICY == CONVGPU_RECENT_FIT) {
+                if (sp < kStack) STK(sp) = (uint8_t)c;
+                ++sp;
+                ru_scan = ru_scan || sp > kStack;
+                AT(s_adm, c) = seq;  // suspension number (scan fallback)
               }
+              ++seq;
             }
-            uint32_t ml, mh;
-            lowmask64(lo, ml, mh);
-            const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
-            uint32_t rsel;
-            if (fl | fh) {  // largest fitting limit, lowest index among equals
-              const uint32_t h = fls64(fl, fh);
-              uint32_t gl, gh;
-              lowmask64(RKB(h, 1), gl, gh);
-              rsel = ffs64(pr_lo & ~gl, pr_hi & ~gh);
-            } else {  // smallest limit, lowest index
-              rsel = ffs64(pr_lo, pr_hi);
-            }
-            sel = RKB(rsel, 2);
-          } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5: most recent suspension
-            if (!ru_scan) {
-              while (sp > 0 && !bit64(pm_lo, pm_hi, STK(sp - 1))) --sp;  // lazy deletion
-              sel = STK(sp - 1);
-            } else {
-              uint32_t best = 0, bs = 0;
+            // DISPATCH has work after a pause with no target (select) or a
+            // FINISH that leaves a target to fill or paused containers
+            dmode = (pause && tnone) || (isX && (target != kNoC || (pm_lo | pm_hi) != 0u));
+            if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true; }
+            const bool adv = !isX && !pause && !badfree;
+            // new state word
+            uint32_t nu = ust;
+            nu = grant ? ((ust & ~kUsedMask) | need | kFirst) : nu;
+            nu = (isF && !badfree) ? ust - r : nu;
+            nu = isX ? (ust & ~kUsedMask) : nu;
+            nu = pause ? (ust | kPaused) : nu;
+            nu = arr ? (vadm ? kAdmitted : 0u) : nu;
+            nu = (adv && !arr) ? nu + kKOne : nu;
+            AT(s_ust, c) = nu;
+            if (arr) AT(s_adm, c) = vadm ? admv : kKeyNone;
+            if (arr || isX) AT(s_nd, c) = arr ? am : t;     // d_1 / finish tick
+            kc = badfree ? kNoC : c;
+            nkc = adv ? (((t + nd) << 6) | c) : kKeyNone;
+            pfk = (adv && !arr) ? ((nu >> kKShift) & 7u) : 0xFFu;
+          }
+        } else {
+          // ====== one DISPATCH step at the triggering tick (R1, R9) ======
+          // A step = [SELECT if there is no fill target] + fill / resume / admit
+          // of the target; an admit keeps the lane in dispatch mode (the
+          // leftover cascades to the next selection, Fig. 3d).
+          const uint32_t t = cur_t;
+          if (target == kNoC) {
+            // ---- SELECT among paused; pm != 0 here ----
+            uint32_t sel;
+            if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
+              sel = ffs64(pm_lo, pm_hi);
+            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
+              // R = #ranks with L <= free (limits sorted by (L, index))
+              uint32_t lo = 0, hi = n;
 #pragma unroll
-              for (uint32_t h = 0; h < 2; ++h) {
-                uint32_t m = h ? pm_hi : pm_lo;
-                while (m) {
-                  const uint32_t b = (uint32_t)(__ffs(m) - 1);
-                  m &= m - 1;
-                  const uint32_t cc = b + 32u * h;
-                  const uint32_t sq = AT(s_adm, cc) + 1u;
-                  if (sq > bs) { bs = sq; best = cc; }
+              for (int it = 0; it < 7; ++it) {
+                if (lo < hi) {
+                  const uint32_t mid = (lo + hi) >> 1;
+                  if (AT(s_L, RKB(mid, 2)) <= free_mem) lo = mid + 1; else hi = mid;
                 }
               }
-              sel = best;
+              uint32_t ml, mh;
+              lowmask64(lo, ml, mh);
+              const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
+              uint32_t rsel;
+              if (fl | fh) {  // largest fitting limit, lowest index among equals
+                const uint32_t h = fls64(fl, fh);
+                uint32_t gl, gh;
+                lowmask64(RKB(h, 1), gl, gh);
+                rsel = ffs64(pr_lo & ~gl, pr_hi & ~gh);
+              } else {  // smallest limit, lowest index
+                rsel = ffs64(pr_lo, pr_hi);
+              }
+              sel = RKB(rsel, 2);
+            } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5: most recent suspension
+              if (!ru_scan) {
+                while (sp > 0 && !bit64(pm_lo, pm_hi, STK(sp - 1))) --sp;  // lazy deletion
+                sel = STK(sp - 1);
+              } else {
+                uint32_t best = 0, bs = 0;
+#pragma unroll
+                for (uint32_t h = 0; h < 2; ++h) {
+                  uint32_t m = h ? pm_hi : pm_lo;
+                  while (m) {
+                    const uint32_t b = (uint32_t)(__ffs(m) - 1);
+                    m &= m - 1;
+                    const uint32_t cc = b + 32u * h;
+                    const uint32_t sq = AT(s_adm, cc) + 1u;
+                    if (sq > bs) { bs = sq; best = cc; }
+                  }
+                }
+                sel = best;
+              }
+            } else {  // RANDOM_FIT (R6)
+              const uint64_t tid = p.tid_base + i;
+              const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
+              const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                         (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+              ++draws;
+              const uint32_t jj = __umulhi(x.x, m);
+              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
             }
-          } else {  // RANDOM_FIT (R6)
-            const uint64_t tid = p.tid_base + i;
-            const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
-            const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
-                                       (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
-            ++draws;
-            const uint32_t jj = __umulhi(x.x, m);
-            sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+            target = sel;
+            a_tg = 0;
+            ++n_sel;
           }
-          target = sel;
-          a_tg = 0;
-          ++n_sel;
-        }
-        {
-          const uint32_t tg = target;
-          const uint32_t Lt = AT(s_L, tg), ut = AT(s_ust, tg), cwt = AT(s_cw, tg),
-                         ndt = AT(s_nd, tg);
-          const uint32_t g = min(free_mem, Lt - a_tg);
-          a_tg += g;
-          free_mem -= g;
-          const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
-          const uint32_t uu = ut & kUsedMask;
-          const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
-          const bool full = a_tg == Lt;                          // admit, cascade
-          used_total += res ? pend : 0u;
-          peak_res = max(peak_res, cap - free_mem);
-          peak_used = max(peak_used, used_total);
-          if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
-          uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
-          nu |= full ? kAdmitted : 0u;
-          AT(s_ust, tg) = nu;
-          if (res) {
-            set64(pm_lo, pm_hi, tg, false);
-            if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
+          {
+            const uint32_t tg = target;
+            const uint32_t Lt = AT(s_L, tg), ut = AT(s_ust, tg), cwt = AT(s_cw, tg),
+                           ndt = AT(s_nd, tg);
+            const uint32_t g = min(free_mem, Lt - a_tg);
+            a_tg += g;
+            free_mem -= g;
+            const uint32_t pend = (cwt & kSizeMask) + ((ut & kFirst) ? 0u : ovh);
+            const uint32_t uu = ut & kUsedMask;
+            const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
+            const bool full = a_tg == Lt;                          // admit, cascade
+            used_total += res ? pend : 0u;
+            peak_res = max(peak_res, cap - free_mem);
+            peak_used = max(peak_used, used_total);
+            if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+            uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
+            nu |= full ? kAdmitted : 0u;
+            AT(s_ust, tg) = nu;
+            if (res) {
+              set64(pm_lo, pm_hi, tg, false);
+              if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
+            }
+            if (full) AT(s_adm, tg) = (t << 6) | rank;
+            rank += full ? 1u : 0u;
+            target = full ? kNoC : target;
+            a_tg = full ? 0u : a_tg;
+            dmode = full && (pm_lo | pm_hi) != 0u;  // another selection follows
+            kc = res ? tg : kNoC;
+            nkc = ((t + ndt) << 6) | tg;
+            pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
           }
-          if (full) AT(s_adm, tg) = (t << 6) | rank;
-          rank += full ? 1u : 0u;
-          target = full ? kNoC : target;
-          a_tg = full ? 0u : a_tg;
-          dmode = full && (pm_lo | pm_hi) != 0u;  // another selection follows
-          kc = res ? tg : kNoC;
-          nkc = ((t + ndt) << 6) | tg;
-          pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
         }
-      }
-      // ---- shared tail: key update, group re-min, op prefetch ----
-      if (kc != kNoC) {
-        AT(s_key, kc) = nkc;
-        regroup(kc);
-        if (pfk != 0xFFu) {  // op k word, delta of op k+1
-          const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
-          if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + off);
-          if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + off + n);
-          pfc = kc;
+        // ---- shared tail: key update, group re-min, op prefetch ----
+        if (kc != kNoC) {
+          AT(s_key, kc) = nkc;
+          regroup(kc);
+          if (pfk != 0xFFu) {  // op k word, delta of op k+1
+            const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
+            if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + off);
+            if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + off + n);
+            pfc = kc;
+          }
         }
+        cp_commit();
       }
-      cp_commit();
-    }
-    if (__all_sync(kFull, !have || tdone) && have) {
+    } while (!__all_sync(kFull, !have || tdone));
+    if (have) {
       epilogue(i);
       i += T;
       have = i < p.count;
