@@ -74,6 +74,14 @@ __device__ __forceinline__ uint32_t smem_addr(const void* p) {
 __device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)), "l"(src) : "memory");
 }
+// predicated forms (one predicated instruction, no divergent branch)
+__device__ __forceinline__ void cp_async4_if(uint32_t* dst, const uint32_t* src, bool on) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q cp.async.ca.shared.global [%0], [%1], 4; }"
+               ::"r"(smem_addr(dst)), "l"(src), "r"((uint32_t)on) : "memory");
+}
+__device__ __forceinline__ void cp_wait0_if(bool on) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q cp.async.wait_group 0; }" ::"r"((uint32_t)on) : "memory");
+}
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
@@ -425,7 +433,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             const uint32_t t = kmin >> 6, c = kmin & 63u;
             cur_t = t;
             cp_wait1();  // every group but the previous iteration's is complete
-            if (c == pf) cp_wait0();
+            cp_wait0_if(c == pf);
             ++events;
             const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
             const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
@@ -594,12 +602,11 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
         if (kc != kNoC) {
           AT(s_key, kc) = nkc;
           regroup(kc);
-          if (pfk != 0xFFu) {  // op k word, delta of op k+1
-            const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
-            if (pfk < K) cp_async4(&AT(s_cw, kc), trace_arg + off);
-            if (pfk + 1 < K) cp_async4(&AT(s_nd, kc), trace_delta + off + n);
-            pfc = kc;
-          }
+          // op k word, delta of op k+1 (pfk = 0xFF: nothing to fetch)
+          const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
+          cp_async4_if(&AT(s_cw, kc), trace_arg + off, pfk < K);
+          cp_async4_if(&AT(s_nd, kc), trace_delta + off + n, pfk + 1 < K);
+          pfc = (pfk != 0xFFu) ? kc : kNoC;
         }
         cp_commit();
       }
