@@ -82,6 +82,10 @@ __device__ __forceinline__ void cp_async4_if(uint32_t* dst, const uint32_t* src,
 __device__ __forceinline__ void cp_wait0_if(bool on) {
   asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q cp.async.wait_group 0; }" ::"r"((uint32_t)on) : "memory");
 }
+__device__ __forceinline__ void sts_if(uint32_t* dst, uint32_t v, bool on) {  // predicated st.shared
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q st.shared.u32 [%0], %1; }"
+               ::"r"(smem_addr(dst)), "r"(v), "r"((uint32_t)on) : "memory");
+}
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
@@ -107,7 +111,8 @@ __device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bo
   hi = on ? (hi | mh) : (hi & ~mh);
 }
 __device__ __forceinline__ uint32_t ffs64(uint32_t lo, uint32_t hi) {  // lowest set bit, 64 if none
-  return lo ? (uint32_t)(__ffs(lo) - 1) : (hi ? 32u + (uint32_t)(__ffs(hi) - 1) : 64u);
+  const uint32_t a = (uint32_t)__ffs(lo), b = (uint32_t)__ffs(hi);  // both always: no branch
+  return a ? a - 1u : (b ? b + 31u : 64u);
 }
 __device__ __forceinline__ uint32_t fls64(uint32_t lo, uint32_t hi) {  // highest set bit
   return hi ? 63u - (uint32_t)__clz(hi) : 31u - (uint32_t)__clz(lo);
@@ -469,20 +474,25 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             rank += vadm ? 1u : 0u;
             n_rej += rej ? 1u : 0u;
             live -= isX ? 1u : 0u;
-            if (pause) {
-              set64(pm_lo, pm_hi, c, true);
-              if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(c, 0), true);
-              if (POLICY == CONVGPU_RECENT_FIT) {
-                if (sp < kStack) STK(sp) = (uint8_t)c;
-                ++sp;
-                ru_scan = ru_scan || sp > kStack;
-                AT(s_adm, c) = seq;  // suspension number (scan fallback)
-              }
-              ++seq;
+            // pause: mark c paused (branch-free: all-ones / zero mask)
+            const uint32_t pmask = pause ? 0xFFFFFFFFu : 0u;
+            pm_lo |= shl_c(1u, c) & pmask;
+            pm_hi |= shl_c(1u, c - 32u) & pmask;
+            if (POLICY == CONVGPU_BEST_FIT) {
+              const uint32_t rc = RKB(c, 0);
+              pr_lo |= shl_c(1u, rc) & pmask;
+              pr_hi |= shl_c(1u, rc - 32u) & pmask;
             }
+            const uint32_t seq0 = seq;
+            if (POLICY == CONVGPU_RECENT_FIT) {
+              if (pause && sp < kStack) STK(sp) = (uint8_t)c;
+              sp += pause ? 1u : 0u;
+              ru_scan = ru_scan || sp > kStack;
+            }
+            seq += pause ? 1u : 0u;
             // DISPATCH has work after a pause with no target (select) or a
             // FINISH that leaves a target to fill or paused containers
-            dmode = (pause && tnone) || (isX && (target != kNoC || (pm_lo | pm_hi) != 0u));
+            dmode = (pause & tnone) | (isX & ((target != kNoC) | ((pm_lo | pm_hi) != 0u)));
             if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true; }
             const bool adv = !isX && !pause && !badfree;
             // new state word
@@ -494,8 +504,10 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             nu = arr ? (vadm ? kAdmitted : 0u) : nu;
             nu = (adv && !arr) ? nu + kKOne : nu;
             AT(s_ust, c) = nu;
-            if (arr) AT(s_adm, c) = vadm ? admv : kKeyNone;
-            if (arr || isX) AT(s_nd, c) = arr ? am : t;     // d_1 / finish tick
+            // admission at arrival; the suspension number (Recent-Fit scan fallback)
+            sts_if(&AT(s_adm, c), arr ? (vadm ? admv : kKeyNone) : seq0,
+                   arr | (POLICY == CONVGPU_RECENT_FIT && pause));
+            sts_if(&AT(s_nd, c), arr ? am : t, arr | isX);  // d_1 / finish tick
             kc = badfree ? kNoC : c;
             nkc = adv ? (((t + nd) << 6) | c) : kKeyNone;
             pfk = (adv && !arr) ? ((nu >> kKShift) & 7u) : 0xFFu;
