@@ -518,12 +518,18 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
           // of the target; an admit keeps the lane in dispatch mode (the
           // leftover cascades to the next selection, Fig. 3d).
           const uint32_t t = cur_t;
-          if (target == kNoC) {
+          if (POLICY == CONVGPU_FIFO) {
+            // ---- SELECT: oldest created paused container (R7);
+            // cheap enough to compute always and keep only with no target ----
+            const bool ns = target == kNoC;
+            const uint32_t sel = ffs64(pm_lo, pm_hi);
+            target = ns ? sel : target;
+            a_tg = ns ? 0u : a_tg;
+            n_sel += ns ? 1u : 0u;
+          } else if (target == kNoC) {
             // ---- SELECT among paused; pm != 0 here ----
             uint32_t sel;
-            if (POLICY == CONVGPU_FIFO) {  // oldest created (R7)
-              sel = ffs64(pm_lo, pm_hi);
-            } else if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
+            if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
               // R = #ranks with L <= free (limits sorted by (L, index))
               uint32_t lo = 0, hi = n;
 #pragma unroll
@@ -610,15 +616,17 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
           }
         }
-        // ---- shared tail: key update, group re-min, op prefetch ----
-        if (kc != kNoC) {
-          AT(s_key, kc) = nkc;
-          regroup(kc);
+        // ---- shared tail: key update, group re-min, op prefetch (branch-free:
+        // with no key change the store is off and group 0 is re-min'ed as is) ----
+        {
+          const uint32_t kcs = kc & 63u;
+          sts_if(&AT(s_key, kcs), nkc, kc != kNoC);
+          regroup(kcs);
           // op k word, delta of op k+1 (pfk = 0xFF: nothing to fetch)
-          const uint32_t off = pfk * n + kc;  // < 2^32: K * n per trace
-          cp_async4_if(&AT(s_cw, kc), trace_arg + off, pfk < K);
-          cp_async4_if(&AT(s_nd, kc), trace_delta + off + n, pfk + 1 < K);
-          pfc = (pfk != 0xFFu) ? kc : kNoC;
+          const uint32_t off = pfk * n + kcs;  // < 2^32: K * n per trace
+          cp_async4_if(&AT(s_cw, kcs), trace_arg + off, pfk < K);
+          cp_async4_if(&AT(s_nd, kcs), trace_delta + off + n, pfk + 1 < K);
+          pfc = (pfk != 0xFFu) ? kcs : kNoC;
         }
         cp_commit();
       }
