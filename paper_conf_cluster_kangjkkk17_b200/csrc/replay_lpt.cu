@@ -530,28 +530,27 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             // ---- SELECT among paused; pm != 0 here ----
             uint32_t sel;
             if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4: shortfall L - 0
-              // R = #ranks with L <= free (limits sorted by (L, index))
+              // R = #ranks with L <= free (limits sorted by (L, index)); a
+              // branch-free binary search (mid clamped once lo == hi)
               uint32_t lo = 0, hi = n;
 #pragma unroll
               for (int it = 0; it < 7; ++it) {
-                if (lo < hi) {
-                  const uint32_t mid = (lo + hi) >> 1;
-                  if (AT(s_L, RKB(mid, 2)) <= free_mem) lo = mid + 1; else hi = mid;
-                }
+                const uint32_t mid = min((lo + hi) >> 1, n - 1u);
+                const bool go = lo < hi, le = AT(s_L, RKB(mid, 2)) <= free_mem;
+                lo = (go & le) ? mid + 1u : lo;
+                hi = (go & !le) ? mid : hi;
               }
               uint32_t ml, mh;
               lowmask64(lo, ml, mh);
               const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
-              uint32_t rsel;
-              if (fl | fh) {  // largest fitting limit, lowest index among equals
-                const uint32_t h = fls64(fl, fh);
-                uint32_t gl, gh;
-                lowmask64(RKB(h, 1), gl, gh);
-                rsel = ffs64(pr_lo & ~gl, pr_hi & ~gh);
-              } else {  // smallest limit, lowest index
-                rsel = ffs64(pr_lo, pr_hi);
-              }
-              sel = RKB(rsel, 2);
+              // largest fitting limit, lowest index among equals; else the
+              // smallest limit, lowest index (both computed, one kept)
+              const uint32_t h = min(fls64(fl, fh), n - 1u);  // in range when nothing fits
+              uint32_t gl, gh;
+              lowmask64(RKB(h, 1), gl, gh);
+              const uint32_t r_fit = ffs64(pr_lo & ~gl, pr_hi & ~gh);
+              const uint32_t r_min = ffs64(pr_lo, pr_hi);
+              sel = RKB((fl | fh) ? r_fit : r_min, 2);
             } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5: most recent suspension
               if (!ru_scan) {
                 while (sp > 0 && !bit64(pm_lo, pm_hi, STK(sp - 1))) --sp;  // lazy deletion
