@@ -158,6 +158,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
 
   // per-trace scheduler ledger (all in registers)
   uint32_t gmin[8];
+  uint32_t piv[8];  // Best-Fit, n = 64: limit at ranks 7, 15, ..., 63 (group maxima)
   uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, seq = 0, rank = 0, draws = 0,
            n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
   uint32_t pm_lo = 0, pm_hi = 0, pr_lo = 0, pr_hi = 0, sp = 0;
@@ -277,6 +278,8 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             }
           }
         }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) piv[j] = v[8 * j + 7] >> 6;
         uint32_t gsr = 0, prevL = 0xFFFFFFFFu;
 #pragma unroll
         for (int r = 0; r < 64; ++r) {
@@ -533,12 +536,25 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
               // R = #ranks with L <= free (limits sorted by (L, index)); a
               // branch-free binary search (mid clamped once lo == hi)
               uint32_t lo = 0, hi = n;
+              if (NF == 64) {
+                // groups of 8 ranks whose maximum fits, then the 8 ranks of the
+                // first group that does not (all 8 loads in flight)
+                uint32_t gc = 0;
 #pragma unroll
-              for (int it = 0; it < 7; ++it) {
-                const uint32_t mid = min((lo + hi) >> 1, n - 1u);
-                const bool go = lo < hi, le = AT(s_L, RKB(mid, 2)) <= free_mem;
-                lo = (go & le) ? mid + 1u : lo;
-                hi = (go & !le) ? mid : hi;
+                for (int j = 0; j < 8; ++j) gc += (piv[j] <= free_mem) ? 1u : 0u;
+                const uint32_t rb = min(gc, 7u) * 8u;
+                uint32_t in = 0;
+#pragma unroll
+                for (uint32_t j = 0; j < 8; ++j) in += (AT(s_L, RKB(rb + j, 2)) <= free_mem) ? 1u : 0u;
+                lo = (gc == 8u) ? 64u : rb + in;
+              } else {
+#pragma unroll
+                for (int it = 0; it < 7; ++it) {
+                  const uint32_t mid = min((lo + hi) >> 1, n - 1u);
+                  const bool go = lo < hi, le = AT(s_L, RKB(mid, 2)) <= free_mem;
+                  lo = (go & le) ? mid + 1u : lo;
+                  hi = (go & !le) ? mid : hi;
+                }
               }
               uint32_t ml, mh;
               lowmask64(lo, ml, mh);
