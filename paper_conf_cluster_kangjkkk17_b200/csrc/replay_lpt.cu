@@ -617,11 +617,15 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
             nu |= full ? kAdmitted : 0u;
             AT(s_ust, tg) = nu;
-            if (res) {
-              set64(pm_lo, pm_hi, tg, false);
-              if (POLICY == CONVGPU_BEST_FIT) set64(pr_lo, pr_hi, RKB(tg, 0), false);
+            const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;  // resumed: no longer paused
+            pm_lo &= ~(shl_c(1u, tg) & rmask);
+            pm_hi &= ~(shl_c(1u, tg - 32u) & rmask);
+            if (POLICY == CONVGPU_BEST_FIT) {
+              const uint32_t rt = RKB(tg, 0);
+              pr_lo &= ~(shl_c(1u, rt) & rmask);
+              pr_hi &= ~(shl_c(1u, rt - 32u) & rmask);
             }
-            if (full) AT(s_adm, tg) = (t << 6) | rank;
+            sts_if(&AT(s_adm, tg), (t << 6) | rank, full);
             rank += full ? 1u : 0u;
             target = full ? kNoC : target;
             a_tg = full ? 0u : a_tg;
