@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define CONVGPU_ABI_VERSION 1
+#define CONVGPU_ABI_VERSION 2
 #define CONVGPU_MAX_CONTAINERS 64u   /* containers per trace */
 #define CONVGPU_MAX_OPS 8u           /* ops per container (K) */
 #define CONVGPU_CAPACITY_LIMIT (1u << 26) /* capacity_mib must be below this */
@@ -216,6 +216,58 @@ int convgpu_replay_host(const convgpu_traces_t *host_traces, uint64_t n,
                         convgpu_summary_t *host_summary, convgpu_stats_t *host_stats,
                         void *device_workspace, size_t workspace_bytes,
                         uint64_t chunk_traces, void *stream);
+
+/* ---- NEXT-3: the wrapper module's size semantics ----------
+ * PAPER.md §III-C: the wrapper intercepts the allocation APIs of Table II
+ * and "calculates adjusted allocate size before checking
+ * available memory size".  convgpu_wrap_ops maps API-level
+ * program records to the op words convgpu_replay consumes:
+ *   MALLOC(bytes = a0 | a1 << 32)          -> ALLOC ceil(bytes / 2^20) MiB
+ *   MALLOC_MANAGED(bytes = a0 | a1 << 32)  -> ALLOC of bytes rounded up to a
+ *                                             multiple of 128 MiB
+ *   MALLOC_PITCH(width a0, height a1)      -> ALLOC of roundup(a0, pitch_align) * a1
+ *                                             bytes
+ *   MALLOC_3D(width a0, height a1, depth a2) -> ALLOC of roundup(a0, pitch_align)
+ *                                             * a1 * a2 bytes (Table II)
+ *   FREE(a0 = op index j of this container) -> FREE of op j's MiB if op j < k is
+ *                                             an allocation not freed before
+ *                                             (the scheduler's address -> size
+ *                                             hash), else FREE of
+ *                                             2^30 - 1 MiB (-> INVALID_FREE)
+ *   MEM_GET_INFO, COMPUTE                  -> NOP (answered from the ledger)
+ *   EXIT (__cudaUnregisterFatBinary)       -> FINISH
+ *   any other code                         -> FINISH if k < n_ops - 1, else NOP
+ *                                             (the replay flags BAD_PROGRAM)
+ * Byte counts become MiB rounded up, saturated at 2^30 - 1 (R13');
+ * products saturate at 2^64 - 1 before rounding.  pitch_align is the device's
+ * pitch granule in bytes (cudaDeviceProp.textureAlignment: 512 on B200, where
+ * cudaMallocPitch returns roundup(width, 512)); 0 = no rounding. */
+typedef enum {
+  CONVGPU_API_MALLOC = 0,
+  CONVGPU_API_MALLOC_MANAGED = 1,
+  CONVGPU_API_MALLOC_PITCH = 2,
+  CONVGPU_API_MALLOC_3D = 3,
+  CONVGPU_API_FREE = 4,
+  CONVGPU_API_MEM_GET_INFO = 5,
+  CONVGPU_API_COMPUTE = 6,
+  CONVGPU_API_EXIT = 7
+} convgpu_api_t;
+
+typedef struct {
+  uint32_t api;        /* convgpu_api_t */
+  uint32_t a0, a1, a2; /* arguments, above */
+} convgpu_api_op_t;    /* 16 bytes */
+
+/* api:    DEVICE, [n][n_ops][n_containers] records, 16-byte aligned (the op_arg
+ *         layout of convgpu_traces_t with a record per op).
+ * op_arg: DEVICE, [n][n_ops][n_containers] u32, written; may be the op_arg of
+ *         a convgpu_traces_t whose other arrays the caller fills.
+ * Caller-owned buffers; asynchronous on `stream` (cudaStream_t or NULL).
+ * Returns 0, -EINVAL (n_containers outside 1..64, n_ops outside 1..8, a
+ * pointer that is NULL, not device memory or api not 16-byte aligned when
+ * n > 0), -ENODEV or -EIO.  n = 0 is a no-op. */
+int convgpu_wrap_ops(const convgpu_api_op_t *api, uint64_t n, uint32_t n_containers,
+                     uint32_t n_ops, uint32_t pitch_align, uint32_t *op_arg, void *stream);
 
 /* Number of kernel launches convgpu_replay and convgpu_generate enqueue per
  * call (convgpu_replay_host: this many per chunk and policy). */

@@ -16,7 +16,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
-_SRC = [os.path.join(_HERE, "oracle.c")]
+_SRC = [os.path.join(_HERE, "oracle.c"), os.path.join(_HERE, "wrapper.c")]
 
 POLICY = {"fifo": 0, "best_fit": 1, "recent_fit": 2, "random_fit": 3}
 NONE32 = 0xFFFFFFFF
@@ -33,7 +33,7 @@ def build(force: bool = False) -> str:
                                "-o", _SO] + _SRC)
         exe = os.path.join(_HERE, "oracle_run")
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-o", exe,
-                               os.path.join(_HERE, "oracle_run.c"), _SRC[0]])
+                               os.path.join(_HERE, "oracle_run.c")] + _SRC)
     return _SO
 
 
@@ -76,6 +76,14 @@ class _Gen(C.Structure):
                 ("ovh", C.c_uint32)]
 
 
+class ApiOp(C.Structure):
+    _fields_ = [("api", C.c_uint32), ("a0", C.c_uint32), ("a1", C.c_uint32), ("a2", C.c_uint32)]
+
+
+API = {"malloc": 0, "malloc_managed": 1, "malloc_pitch": 2, "malloc_3d": 3, "free": 4,
+       "mem_get_info": 5, "compute": 6, "exit": 7}
+API_DTYPE = np.dtype([("api", np.uint32), ("a0", np.uint32), ("a1", np.uint32), ("a2", np.uint32)])
+
 _lib = None
 
 
@@ -99,6 +107,12 @@ def lib():
                                        u32p, u32p, C.c_uint32, C.c_int, C.c_uint64,
                                        C.c_uint64, C.c_uint32, C.c_int, C.POINTER(Stats),
                                        u32p, u64p, u32p, u32p, u8p, u32p, u32p]
+        L.orc_wrap_bytes.argtypes = [C.POINTER(ApiOp), C.c_uint32]
+        L.orc_wrap_bytes.restype = C.c_uint64
+        L.orc_wrap_mib.argtypes = [C.c_uint64]
+        L.orc_wrap_mib.restype = C.c_uint32
+        L.orc_wrap_program.argtypes = [C.POINTER(ApiOp), C.c_uint32, C.c_uint32, u32p]
+        L.orc_wrap_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, C.c_void_p, C.c_uint32, u32p]
         _lib = L
     return _lib
 
@@ -232,3 +246,31 @@ def replay_batch(b, cap, policy, tid_base=0, rand_seed=0, ovh=0, check=False, fu
     res = _pack(o, st)
     res["rc"] = rc
     return res
+
+
+# ---- NEXT-3: wrapper-side size semantics (oracle/wrapper.c) ----
+def wrap_bytes(api, a0=0, a1=0, a2=0, pitch_align=512) -> int:
+    op = ApiOp(API[api] if isinstance(api, str) else api, a0, a1, a2)
+    return int(lib().orc_wrap_bytes(C.byref(op), pitch_align))
+
+
+def wrap_mib(nbytes: int) -> int:
+    return int(lib().orc_wrap_mib(nbytes))
+
+
+def wrap_program(ops, pitch_align=512):
+    """ops: list of (api, a0, a1, a2) for one container -> list of op words."""
+    K = len(ops)
+    arr = (ApiOp * K)(*[ApiOp(API[o[0]] if isinstance(o[0], str) else o[0], *o[1:]) for o in ops])
+    out = np.zeros(K, np.uint32)
+    lib().orc_wrap_program(arr, K, pitch_align, _p(out))
+    return [int(x) for x in out]
+
+
+def wrap_batch(api, pitch_align=512):
+    """api: structured array API_DTYPE [count, K, n] -> op_arg uint32 [count, K, n]."""
+    api = np.ascontiguousarray(api, API_DTYPE)
+    count, K, n = api.shape
+    out = np.zeros((count, K, n), np.uint32)
+    lib().orc_wrap_batch(n, K, count, api.ctypes.data, pitch_align, _p(out))
+    return out

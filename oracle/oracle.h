@@ -116,6 +116,36 @@ int orc_replay_batch(uint32_t n, uint32_t K, uint64_t count,
                      uint32_t *cnt_u32x2, uint32_t *admit_tick,
                      uint8_t *admit_rank, uint32_t *wait, uint32_t *finish);
 
+/* ---- NEXT-3: wrapper-side size semantics (oracle/wrapper.c) ------------
+ * The wrapper module sees CUDA API calls and "calculates adjusted allocate
+ * size before checking available memory size"; Table II
+ * lists the covered APIs.  An API-level program record per
+ * (container, op) is mapped to the scheduler's op word. */
+enum {
+  ORC_API_MALLOC = 0,         /* cudaMalloc / cuMemAlloc(bytes = a0 | a1 << 32) */
+  ORC_API_MALLOC_MANAGED = 1, /* cudaMallocManaged(bytes): multiple of 128 MiB */
+  ORC_API_MALLOC_PITCH = 2,   /* cudaMallocPitch(width a0, height a1): pitch * height */
+  ORC_API_MALLOC_3D = 3,      /* cudaMalloc3D(width a0, height a1, depth a2) */
+  ORC_API_FREE = 4,           /* cudaFree of the allocation made by op a0 of this container */
+  ORC_API_MEM_GET_INFO = 5,   /* cudaMemGetInfo: answered from the ledger, no memory effect */
+  ORC_API_COMPUTE = 6,        /* work without memory calls */
+  ORC_API_EXIT = 7            /* __cudaUnregisterFatBinary */
+};
+typedef struct {
+  uint32_t api, a0, a1, a2;
+} orc_api_op_t;
+/* Bytes an allocation API really takes (saturating at 2^64 - 1); 0 for a
+ * non-allocation API.  pitch_align = the device's pitch granule in bytes. */
+uint64_t orc_wrap_bytes(const orc_api_op_t *op, uint32_t pitch_align);
+/* The scheduler's unit is MiB: ceil(bytes / 2^20), saturated to 2^30 - 1. */
+uint32_t orc_wrap_mib(uint64_t bytes);
+/* One container's program of K API records -> K op words. */
+void orc_wrap_program(const orc_api_op_t *ops, uint32_t K, uint32_t pitch_align,
+                      uint32_t *op_words);
+/* A batch laid out like the C-ABI: api[(i*K + k)*n + c] -> arg[(i*K + k)*n + c]. */
+void orc_wrap_batch(uint32_t n, uint32_t K, uint64_t count, const orc_api_op_t *api,
+                    uint32_t pitch_align, uint32_t *arg);
+
 #ifdef __cplusplus
 }
 #endif

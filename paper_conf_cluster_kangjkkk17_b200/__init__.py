@@ -73,8 +73,14 @@ class BuffersT(C.Structure):
 
 
 EXPORTS = ("convgpu_replay", "convgpu_generate", "convgpu_replay_host",
-           "convgpu_replay_host_workspace", "convgpu_launches_per_call", "convgpu_strerror",
-           "convgpu_abi_version")
+           "convgpu_replay_host_workspace", "convgpu_wrap_ops", "convgpu_launches_per_call",
+           "convgpu_strerror", "convgpu_abi_version")
+
+# NEXT-3 API records (include/convgpu.h convgpu_api_t / convgpu_api_op_t)
+API = {"malloc": 0, "malloc_managed": 1, "malloc_pitch": 2, "malloc_3d": 3, "free": 4,
+       "mem_get_info": 5, "compute": 6, "exit": 7}
+API_DTYPE = np.dtype([("api", np.uint32), ("a0", np.uint32), ("a1", np.uint32), ("a2", np.uint32)])
+B200_PITCH_ALIGN = 512  # cudaDeviceProp.textureAlignment = cudaMallocPitch granule on B200
 
 _lib = None
 
@@ -96,6 +102,8 @@ def lib():
         L.convgpu_replay_host_workspace.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64,
                                                     C.c_uint32]
         L.convgpu_replay_host_workspace.restype = C.c_size_t
+        L.convgpu_wrap_ops.argtypes = [C.c_void_p, C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32,
+                                       C.c_void_p, C.c_void_p]
         L.convgpu_strerror.argtypes = [C.c_int]
         L.convgpu_strerror.restype = C.c_char_p
         _lib = L
@@ -193,6 +201,21 @@ def generate(g, trace_id_base: int, count: int, device="cuda", out: Optional[Tra
     _check(lib().convgpu_generate(C.byref(gen_params_struct(g)), trace_id_base, count,
                                   C.byref(buf), _stream_handle(stream)), "convgpu_generate")
     return t
+
+
+def wrap_ops(api, n: int, K: int, pitch_align: int = B200_PITCH_ALIGN, out=None, stream=None):
+    """NEXT-3: map API-level records to scheduler op words on the device
+    (convgpu_wrap_ops).  api: int32 tensor [N, K, n, 4] (convgpu_api_op_t
+    records) on the GPU; returns (or fills) the int32 op_arg tensor [N, K, n]."""
+    import torch
+    if api.dim() != 4 or api.shape[1] != K or api.shape[2] != n or api.shape[3] != 4:
+        raise ConvgpuError("api must be [N, K, n, 4] int32")
+    N = api.shape[0]
+    if out is None:
+        out = torch.empty((N, K, n), dtype=torch.int32, device=api.device)
+    _check(lib().convgpu_wrap_ops(api.data_ptr(), N, n, K, pitch_align, out.data_ptr(),
+                                  _stream_handle(stream)), "convgpu_wrap_ops")
+    return out
 
 
 @dataclass

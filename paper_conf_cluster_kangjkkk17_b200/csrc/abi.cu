@@ -165,6 +165,19 @@ int convgpu_generate(const convgpu_gen_params_t* p, uint64_t trace_id_base, uint
   return e == cudaSuccess ? 0 : fail_cuda(e, "generate launch");
 }
 
+int convgpu_wrap_ops(const convgpu_api_op_t* api, uint64_t n, uint32_t n_containers, uint32_t n_ops,
+                     uint32_t pitch_align, uint32_t* op_arg, void* stream) {
+  if (n_containers < 1 || n_containers > CONVGPU_MAX_CONTAINERS) return -EINVAL;
+  if (n_ops < 1 || n_ops > CONVGPU_MAX_OPS) return -EINVAL;
+  int rc = check_device();
+  if (rc) return rc;
+  if (n == 0) return 0;
+  if (!is_device_ptr(api) || !is_device_ptr(op_arg) || !aligned16(api)) return -EINVAL;
+  cudaError_t e = convgpu::launch_wrap(reinterpret_cast<const uint4*>(api), n, n_containers, n_ops,
+                                       pitch_align, op_arg, (cudaStream_t)stream);
+  return e == cudaSuccess ? 0 : fail_cuda(e, "wrap launch");
+}
+
 // ---------------------------------------------------------------- host e2e
 // Workspace layout (256-B aligned pieces): 2 x {arrival, limit, delta, arg}
 // chunk buffers, 2 x n_policies summary chunks, n_policies stats structs.

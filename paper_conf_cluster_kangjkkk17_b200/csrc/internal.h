@@ -39,4 +39,7 @@ struct GenArgs {
 
 cudaError_t launch_generate(const GenArgs& a, cudaStream_t stream);
 
+cudaError_t launch_wrap(const uint4* api, uint64_t count, uint32_t n, uint32_t K, uint32_t pitch,
+                        uint32_t* arg, cudaStream_t stream);
+
 }  // namespace convgpu

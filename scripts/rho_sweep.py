@@ -7,7 +7,13 @@ For rho = 1..8 (declared limits scaled by 15*rho/7, so E[sum L]/cap = rho),
 (statistics only, no per-trace outputs).  Writes per-(rho, policy, seed) means
 and the seed spread to profiles/<tag>_rho_sweep.json and a markdown table.
 
-  python scripts/rho_sweep.py [--traces 1000000] [--seeds 32] [--tag r01]
+  python scripts/rho_sweep.py [--traces 1000000] [--seeds 32] [--lit-seeds 8] [--tag r01]
+
+NEXT-1: every point is also replayed under the literal
+re-select-on-every-release reading R1-LIT (warp-per-trace kernel), all four
+policies (Random-Fit seeds 0..lit_seeds-1), recording the deadlock share per
+policy and rho (the paper's no-deadlock claim, P:7, under the other reading)
+and the means over the traces that did not deadlock.
 
 Sharding over G GPUs (torchrun) splits each point's trace-id range; on one GPU
 the points run back to back.  Parity of the sweep's kernels against the
@@ -30,6 +36,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--traces", type=int, default=1_000_000)
     ap.add_argument("--seeds", type=int, default=32)
+    ap.add_argument("--lit-seeds", type=int, default=8)
     ap.add_argument("--tag", default="r01")
     a = ap.parse_args()
     import torch
@@ -61,6 +68,37 @@ def main():
                          "max_peak_reserved_mib": st["max_peak_reserved"],
                          "flag_count": st["flag_count"], "digest_sum": "%016x" % st["digest_sum"],
                          "events": st["events"], "ms": e0.elapsed_time(e1)})
+    # R1-LIT (NEXT-1): deadlock share per policy and rho
+    lit_rows = []
+    for rho in range(1, 9):
+        w = W.rho_sweep(rho, n_traces=a.traces)
+        buf = cg.generate(w.gen, 0, a.traces, device=dev, out=buf)
+        runs = [("fifo", 0), ("best_fit", 0), ("recent_fit", 0)] + \
+               [("random_fit", s) for s in range(a.lit_seeds)]
+        for pol, seed in runs:
+            out = cg.alloc_out(a.traces, w.gen.n, device=dev, full=False, summary=False)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            cg.replay(buf, w.cap, pol + "+literal", out, rand_seed=seed)
+            e1.record()
+            torch.cuda.synchronize()
+            st = cg.stats_dict(out.stats_np())
+            ok = st["traces"] - st["flag_count"][0]  # deadlocked traces report zeros
+            lit_rows.append({"rho": rho, "policy": pol, "seed": seed,
+                             "deadlock_share": st["flag_count"][0] / st["traces"],
+                             "mean_makespan_s_ok": st["sum_makespan"] / max(ok, 1) / 1000.0,
+                             "mean_wait_s_ok": st["sum_wait"] / (max(ok, 1) * w.gen.n) / 1000.0,
+                             "digest_sum": "%016x" % st["digest_sum"], "events": st["events"],
+                             "ms": e0.elapsed_time(e1)})
+    lit_table = []
+    for rho in range(1, 9):
+        line = {"rho": rho}
+        for pol in ("fifo", "best_fit", "recent_fit", "random_fit"):
+            rr = [x for x in lit_rows if x["rho"] == rho and x["policy"] == pol]
+            line[pol] = {"deadlock_share": statistics.mean(x["deadlock_share"] for x in rr),
+                         "mean_makespan_s_ok": statistics.mean(x["mean_makespan_s_ok"] for x in rr),
+                         "mean_wait_s_ok": statistics.mean(x["mean_wait_s_ok"] for x in rr)}
+        lit_table.append(line)
     table = []
     for rho in range(1, 9):
         line = {"rho": rho}
@@ -81,7 +119,12 @@ def main():
     doc = {"config": "BASELINE configs[4]", "traces_per_point": a.traces, "seeds": a.seeds,
            "capacity_mib": 184320, "containers": 64, "unit_time": "s (1 tick = 1 ms)",
            "replay_events": ev, "replay_ms": ms, "events_per_s": ev / (ms / 1e3),
-           "wall_s": time.time() - t_all, "table": table, "runs": rows}
+           "wall_s": time.time() - t_all, "table": table, "runs": rows,
+           "literal": {"reading": "R1-LIT (DESIGN.md §6.5, NEXT-1)", "seeds": a.lit_seeds,
+                       "events": sum(x["events"] for x in lit_rows),
+                       "events_per_s": sum(x["events"] for x in lit_rows) /
+                       (sum(x["ms"] for x in lit_rows) / 1e3),
+                       "table": lit_table, "runs": lit_rows}}
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     with open(os.path.join(ROOT, "gpurun_out", f"{a.tag}_rho_sweep.json")
               if os.path.isdir(os.path.join(ROOT, "gpurun_out")) else
@@ -95,6 +138,10 @@ def main():
               f"{r['makespan_mean']:.2f}±{r['makespan_sd']:.3f} [{r['makespan_min']:.2f},"
               f"{r['makespan_max']:.2f}] / {r['wait_mean']:.2f} | {l['deadlocks']}")
     print(f"{ev:.3e} events in {ms / 1e3:.2f} s of replay = {ev / (ms / 1e3):.3e} events/s")
+    print("R1-LIT deadlock share: rho | FIFO | BF | RU | Rand")
+    for l in lit_table:
+        print(f"{l['rho']} | " + " | ".join(f"{l[p]['deadlock_share']:.4f}" for p in
+                                            ("fifo", "best_fit", "recent_fit", "random_fit")))
 
 
 if __name__ == "__main__":

@@ -212,3 +212,76 @@ def random_batch(seed: int, count: int, n: int, K: int, cap: int, ovh: int = 0,
 
 def with_fields(w: Workload, **kw) -> Workload:
     return dataclasses.replace(w, **kw)
+
+
+# ---------------------------------------------------------------------------
+# NEXT-3: API-level programs (the wrapper module's input, PAPER.md P:104-110,
+# Table II).  Records [count, K, n] of (api, a0, a1, a2) in the
+# convgpu_api_op_t layout; API codes as in include/convgpu.h.  Input recipe
+# only: random API calls and arguments, none of the size arithmetic.
+API_MALLOC, API_MANAGED, API_PITCH, API_3D, API_FREE, API_MEMINFO, API_COMPUTE, API_EXIT = range(8)
+API_RECORD = np.dtype([("api", np.uint32), ("a0", np.uint32), ("a1", np.uint32), ("a2", np.uint32)])
+
+
+def _api_bytes(rng, scale_mib: int):
+    """A byte count of log-uniform magnitude up to ~scale_mib MiB, as (lo, hi)."""
+    top = max(int(scale_mib) << 20, 1)
+    b = int(np.exp(rng.uniform(0.0, np.log(top + 1)))) - 1
+    if rng.random() < 0.1:
+        b = int(rng.choice([0, 1, (1 << 20) - 1, 1 << 20, (1 << 20) + 1, (128 << 20) - 1,
+                            128 << 20, (128 << 20) + 1]))
+    return b & 0xFFFFFFFF, b >> 32
+
+
+def random_api_batch(seed: int, count: int, n: int, K: int, mode: str = "valid",
+                     scale_mib: int = 4096) -> np.ndarray:
+    """Seeded API-level programs.  'valid': allocations through the four
+    allocation APIs, cudaFree of earlier allocations, cudaMemGetInfo /
+    compute records, EXIT last.  'mixed': also frees naming later ops,
+    non-allocations or freed allocations, unknown API codes anywhere, huge
+    (saturating) arguments and a missing EXIT."""
+    rng = np.random.default_rng(seed)
+    out = np.zeros((count, K, n), API_RECORD)
+    for i in range(count):
+        for c in range(n):
+            allocs = []
+            for k in range(K):
+                rec = [API_COMPUTE, 0, 0, 0]
+                last = k == K - 1
+                r = rng.random()
+                if last and (mode == "valid" or rng.random() < 0.9):
+                    rec = [API_EXIT, 0, 0, 0]
+                elif r < 0.2:
+                    lo, hi = _api_bytes(rng, scale_mib)
+                    rec = [API_MALLOC, lo, hi, int(rng.integers(0, 1 << 32))]
+                elif r < 0.35:
+                    lo, hi = _api_bytes(rng, scale_mib)
+                    rec = [API_MANAGED, lo, hi, 0]
+                elif r < 0.6:
+                    # moderate extents (<= 1 GiB); 'mixed' also draws full 32-bit ones
+                    wide = mode != "valid"
+                    big = lambda b: int(rng.integers(0, 1 << 32)) if wide and rng.random() < 0.2 \
+                        else int(rng.integers(0, 1 << b))
+                    if r < 0.5:
+                        rec = [API_PITCH, big(16), big(14), int(rng.integers(0, 1 << 32))]
+                    else:
+                        rec = [API_3D, big(14), big(10), big(6)]
+                elif r < 0.8:
+                    live = [j for j in allocs]
+                    if mode == "valid":
+                        if live:
+                            j = live[int(rng.integers(0, len(live)))]
+                            allocs.remove(j)
+                            rec = [API_FREE, j, 0, 0]
+                        else:
+                            rec = [API_MEMINFO, 0, 0, 0]
+                    else:
+                        rec = [API_FREE, int(rng.integers(0, K + 2)), 0, 0]
+                elif r < 0.9:
+                    rec = [API_MEMINFO, 0, 0, 0]
+                if mode != "valid" and rng.random() < 0.05:
+                    rec[0] = int(rng.choice([8, 9, 15, 0xFFFFFFFF]))
+                if rec[0] <= API_3D and rec[0] < 8:
+                    allocs.append(k)
+                out[i, k, c] = tuple(rec)
+    return out
