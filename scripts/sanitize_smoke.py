@@ -1,5 +1,6 @@
 """Small replay of every kernel variant / policy (incl. the literal reading)
-for compute-sanitizer runs: memcheck, racecheck, synccheck, initcheck."""
+and the NEXT-3 wrapper kernel for compute-sanitizer runs: memcheck,
+racecheck, synccheck, initcheck."""
 import os
 import sys
 
@@ -27,5 +28,14 @@ tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
 for kernel in ("warp", "lane"):
     for pol in W.POLICIES:
         cg.replay(tr, 16, pol, cg.alloc_out(200, 7), ovh=2, kernel=kernel)
+torch.cuda.synchronize()
+# NEXT-3 wrapper kernel: the n = 64 / K = 4 fast path, K = 4 and generic shapes
+import numpy as np  # noqa: E402
+for (N, n, K) in ((300, 64, 4), (97, 5, 4), (50, 7, 8)):
+    api = W.random_api_batch(9, N, n, K, "mixed")
+    t = torch.from_numpy(np.ascontiguousarray(api).view(np.uint32).reshape(N, K, n, 4)
+                         .view(np.int32)).cuda()
+    for pitch in (512, 1000, 0):
+        cg.wrap_ops(t, n, K, pitch_align=pitch)
 torch.cuda.synchronize()
 print("sanitize smoke done")
