@@ -46,5 +46,48 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return SO
 
 
+# ---- NEXT-4: the live control plane (native, host side) --------------------
+CTL = os.path.join(CSRC, "ctl")
+DAEMON = os.path.join(PKG, "convgpud")
+SHIM = os.path.join(PKG, "libconvgpu_shim.so")
+CXX = os.environ.get("CXX", "g++")
+CTL_HDR = [os.path.join(ROOT, "include", "convgpu_ctl.h"), os.path.join(CTL, "sched.hpp")]
+
+
+def _run(cmd, what):
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError(f"{what} failed ({r.returncode})")
+
+
+def _older(out, srcs):
+    return not os.path.exists(out) or any(os.path.getmtime(s) > os.path.getmtime(out) for s in srcs)
+
+
+def build_ctl(force: bool = False) -> tuple:
+    """convgpud (scheduler daemon) and libconvgpu_shim.so (LD_PRELOAD wrapper
+    module, linked against nothing CUDA: it resolves the real CUDA entry points
+    with dlsym(RTLD_NEXT) at run time)."""
+    dsrc = [os.path.join(CTL, "convgpud.cpp"), os.path.join(CTL, "sched.cpp")]
+    if force or _older(DAEMON, dsrc + CTL_HDR):
+        _run([CXX, "-O2", "-std=c++17", "-Wall", "-Wextra", "-I" + os.path.join(ROOT, "include"),
+              "-o", DAEMON + ".tmp"] + dsrc,
+             "convgpud build")
+        os.replace(DAEMON + ".tmp", DAEMON)
+    ssrc = [os.path.join(CTL, "shim.cpp")]
+    if os.path.exists(ssrc[0]) and (force or _older(SHIM, ssrc + CTL_HDR)):
+        # no C++ runtime, hidden by default: only the CUDA entry points are exported
+        _run([CXX, "-O2", "-std=c++17", "-Wall", "-Wextra", "-fPIC", "-shared",
+              "-fno-exceptions", "-fno-rtti", "-fno-threadsafe-statics", "-nostdlib++",
+              "-fvisibility=hidden",
+              "-I/usr/local/cuda/include", "-I" + os.path.join(ROOT, "include"),
+              "-o", SHIM + ".tmp"] + ssrc + ["-ldl", "-lpthread"],
+             "shim build")
+        os.replace(SHIM + ".tmp", SHIM)
+    return DAEMON, SHIM
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose=True))
+    print(build_ctl(force="--force" in sys.argv))
