@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--workload", default="c2", choices=["c1", "c2", "mimic"])
     ap.add_argument("--traces", type=int, default=None, help="traces per GPU (default: config)")
     ap.add_argument("--outputs", default="full", choices=["full", "summary"])
-    ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane"])
+    ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane", "lane16"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -277,10 +277,13 @@ def run_ours(args, rank, local_rank, world):
     per_trace_events = n * (1 + K)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
 
-    def kernel_of(p):  # the rule of abi.cu auto_variant
+    def kernel_of(p):  # the rule of abi.cu launch_any / auto_variant
         if args.kernel != "auto":
             return args.kernel
-        return "lane" if Nr >= sms * 2 * 64 * 4 else "warp"
+        if Nr < sms * 2 * 64 * 4:
+            return "warp"
+        return "lane16" if (full and n == 64 and K == 4) else "lane"
+    launches_per_replay = {p: 2 if kernel_of(p) == "lane16" else 1 for p in POLICIES}
     kernel_used = ",".join(sorted({kernel_of(p) for p in POLICIES}))
     # correctness of the timed work: every timed launch replayed every trace
     last = args.warmup + args.steps - 1
@@ -338,7 +341,7 @@ def run_ours(args, rank, local_rank, world):
             "gen_ms": gen_ms,
             "gen_write_gbs": Nr * in_b / (gen_ms / 1e3) / 1e9,
             "roofline": roofline,
-            "gpu_launches": args.steps * len(POLICIES) * cg.lib().convgpu_launches_per_call(),
+            "gpu_launches": args.steps * sum(launches_per_replay.values()),
             "clocks": clocks,
         }
 

@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define CONVGPU_ABI_VERSION 2
+#define CONVGPU_ABI_VERSION 3
 #define CONVGPU_MAX_CONTAINERS 64u   /* containers per trace */
 #define CONVGPU_MAX_OPS 8u           /* ops per container (K) */
 #define CONVGPU_CAPACITY_LIMIT (1u << 26) /* capacity_mib must be below this */
@@ -110,7 +110,16 @@ typedef struct {
 enum {
   CONVGPU_KERNEL_AUTO = 0,
   CONVGPU_KERNEL_WARP_PER_TRACE = 1, /* one warp per trace, TMA-staged trace */
-  CONVGPU_KERNEL_LANE_PER_TRACE = 2  /* one lane per trace, 32 traces per warp */
+  CONVGPU_KERNEL_LANE_PER_TRACE = 2, /* one lane per trace, 32 traces per warp */
+  CONVGPU_KERNEL_LANE_COMPACT = 3    /* one lane per trace, 16-bit packed state, up to
+                                        8 warps per SM; needs n_containers = 64, n_ops = 4,
+                                        out->admit_tick != NULL (it holds admissions during
+                                        the replay) and 16-byte aligned arrays / outputs,
+                                        else -EINVAL.  Traces whose limits exceed 0xFFFE
+                                        MiB, deltas 0xFFFF ticks or horizon 2^25 are
+                                        replayed by a second, 32-bit lane-per-trace launch.
+                                        AUTO picks it whenever the lane kernel would run
+                                        and these conditions hold. */
 };
 
 /* Per-trace summary, 40 bytes. */
@@ -156,7 +165,7 @@ typedef struct {
  * (no-op).
  * Errors: -EINVAL for NULL traces/out/arrays, n_containers or n_ops out of
  * range, policy out of range, capacity out of range, overhead out of range,
- * kernel_variant > 2, host pointers, range_digest without range_size; -ENODEV;
+ * kernel_variant > 3 (or 3 without its conditions), host pointers, range_digest without range_size; -ENODEV;
  * -EIO (launch failure).
  */
 int convgpu_replay(const convgpu_traces_t *traces, uint64_t n, uint32_t capacity_mib,
@@ -269,8 +278,10 @@ typedef struct {
 int convgpu_wrap_ops(const convgpu_api_op_t *api, uint64_t n, uint32_t n_containers,
                      uint32_t n_ops, uint32_t pitch_align, uint32_t *op_arg, void *stream);
 
-/* Number of kernel launches convgpu_replay and convgpu_generate enqueue per
- * call (convgpu_replay_host: this many per chunk and policy). */
+/* Upper bound on the kernel launches convgpu_replay enqueues per call (the
+ * compact lane kernel is followed by its 32-bit fallback pass; every other
+ * variant launches once; convgpu_generate launches once;
+ * convgpu_replay_host: this many per chunk and policy). */
 int convgpu_launches_per_call(void);
 
 /* Human-readable text for a return code (thread-local CUDA text for -EIO). */

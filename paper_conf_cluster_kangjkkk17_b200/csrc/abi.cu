@@ -6,6 +6,7 @@
 #include <errno.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include "convgpu.h"
@@ -53,11 +54,12 @@ int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
   if (t->n_ops < 1 || t->n_ops > CONVGPU_MAX_OPS) return -EINVAL;
   if (policy < 0 || (policy & ~(0xFF | CONVGPU_DISPATCH_LITERAL)) || (policy & 0xFF) > 3)
     return -EINVAL;
-  if ((policy & CONVGPU_DISPATCH_LITERAL) && t->kernel_variant == CONVGPU_KERNEL_LANE_PER_TRACE)
+  if ((policy & CONVGPU_DISPATCH_LITERAL) && (t->kernel_variant == CONVGPU_KERNEL_LANE_PER_TRACE ||
+                                               t->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT))
     return -EINVAL;
   if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
   if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
-  if (t->kernel_variant > CONVGPU_KERNEL_LANE_PER_TRACE) return -EINVAL;
+  if (t->kernel_variant > CONVGPU_KERNEL_LANE_COMPACT) return -EINVAL;
   return 0;
 }
 
@@ -73,6 +75,7 @@ convgpu::ReplayArgs make_args(const convgpu_traces_t* t, uint64_t n, uint32_t ca
   a.n = t->n_containers; a.K = t->n_ops;
   a.tid_base = t->trace_id_base; a.seed = t->rand_seed;
   a.ovh = t->ctx_overhead_mib; a.cap = cap; a.count = n;
+  if (const char* s = getenv("CONVGPU_PER_SM_CAP")) a.per_sm_cap = (uint32_t)strtoul(s, nullptr, 10);
   return a;
 }
 
@@ -97,7 +100,15 @@ cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cuda
   a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.wait) &&
                 aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
   if (policy & CONVGPU_DISPATCH_LITERAL) variant = CONVGPU_KERNEL_WARP_PER_TRACE;
-  if (variant == CONVGPU_KERNEL_AUTO) variant = auto_variant(a.count, policy);
+  if (variant == CONVGPU_KERNEL_AUTO) {
+    variant = auto_variant(a.count, policy);
+    if (variant == CONVGPU_KERNEL_LANE_PER_TRACE && convgpu::lpt16_supported(a))
+      variant = CONVGPU_KERNEL_LANE_COMPACT;
+  }
+  if (variant == CONVGPU_KERNEL_LANE_COMPACT) {
+    if (!convgpu::lpt16_supported(a)) return cudaErrorInvalidValue;  // -EINVAL, see convgpu_replay
+    return convgpu::launch_replay_lpt16(a, policy, s);
+  }
   if (variant == CONVGPU_KERNEL_LANE_PER_TRACE) return convgpu::launch_replay_lpt(a, policy, s);
   return convgpu::launch_replay(a, policy, use_bulk(a), s);
 }
@@ -108,7 +119,7 @@ extern "C" {
 
 int convgpu_abi_version(void) { return CONVGPU_ABI_VERSION; }
 
-int convgpu_launches_per_call(void) { return 1; }
+int convgpu_launches_per_call(void) { return 2; }  // compact lane kernel + its 32-bit fallback pass
 
 const char* convgpu_strerror(int rc) {
   switch (rc) {
@@ -126,6 +137,9 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   if (rc) return rc;
   if (!out) return -EINVAL;
   if (out->range_digest && out->range_size == 0) return -EINVAL;
+  if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT &&
+      (traces->n_containers != 64 || traces->n_ops != 4 || !out->admit_tick))
+    return -EINVAL;
   if (n == 0) return 0;  // no-op: array pointers may be NULL
   if ((rc = validate_arrays(traces))) return rc;
   if ((rc = check_device())) return rc;
@@ -142,6 +156,11 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   a.wait = out->wait; a.finish = out->finish;
   a.summary = out->summary; a.stats = out->stats;
   a.range_digest = out->range_digest; a.range_size = out->range_size;
+  if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT) {
+    a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.wait) &&
+                  aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
+    if (!convgpu::lpt16_supported(a)) return -EINVAL;
+  }
   cudaError_t e = launch_any(a, policy, traces->kernel_variant, (cudaStream_t)out->stream);
   return e == cudaSuccess ? 0 : fail_cuda(e, "replay launch");
 }
@@ -180,7 +199,8 @@ int convgpu_wrap_ops(const convgpu_api_op_t* api, uint64_t n, uint32_t n_contain
 
 // ---------------------------------------------------------------- host e2e
 // Workspace layout (256-B aligned pieces): 2 x {arrival, limit, delta, arg}
-// chunk buffers, 2 x n_policies summary chunks, n_policies stats structs.
+// chunk buffers, 2 x n_policies summary chunks, n_policies stats structs, one
+// chunk of per-container admission scratch.
 static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops, uint64_t chunk,
@@ -188,7 +208,7 @@ size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops, uint
   const size_t cn = align256(chunk * n_containers * 4);
   const size_t ckn = align256(chunk * n_containers * n_ops * 4);
   return 2 * (2 * cn + 2 * ckn) + 2 * (size_t)n_policies * align256(chunk * sizeof(convgpu_summary_t)) +
-         (size_t)n_policies * align256(sizeof(convgpu_stats_t));
+         (size_t)n_policies * align256(sizeof(convgpu_stats_t)) + cn;  // + admission scratch
 }
 
 int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, uint32_t policy_mask,
@@ -222,6 +242,9 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     for (int q = 0; q < np; ++q) { sum[b][q] = (convgpu_summary_t*)w; w += sb; }
   convgpu_stats_t* dstats = (convgpu_stats_t*)w;  // [np], 256-B apart
   const size_t stb = align256(sizeof(convgpu_stats_t));
+  // per-container admissions of the chunk being replayed: the compact lane
+  // kernel keeps them here during a replay (launches are stream-ordered)
+  uint32_t* adm_scratch = (uint32_t*)(w + (size_t)np * stb);
 
   cudaStream_t copy = nullptr;
   cudaEvent_t h2d[2] = {nullptr, nullptr}, kdone[2] = {nullptr, nullptr};
@@ -263,6 +286,7 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
+      a.admit_tick = adm_scratch;
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
       e = launch_any(a, pols[q], ht->kernel_variant, cs);
     }

@@ -25,11 +25,18 @@ struct ReplayArgs {
   uint64_t* range_digest;
   uint64_t range_size;
   uint64_t grid_override;  // 0 = occupancy-sized persistent grid
+  uint32_t per_sm_cap;     // tuning knob (env CONVGPU_PER_SM_CAP): at most this many CTAs per SM
   uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
+  uint32_t only_marked;    // lane kernel: replay only traces with admit_tick[i*n] == kLpt16Mark
 };
+
+// admit_tick[i*n] of a trace the compact kernel left to the 32-bit lane kernel
+constexpr uint32_t kLpt16Mark = 0xFFFFFFFEu;
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream);
 cudaError_t launch_replay_lpt(const ReplayArgs& a, int policy, cudaStream_t stream);
+bool lpt16_supported(const ReplayArgs& a);
+cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream);
 
 struct GenArgs {
   convgpu_gen_params_t p;

@@ -1,0 +1,66 @@
+// lpt_util.cuh — small PTX helpers shared by the lane-per-trace replay
+// kernels (replay_lpt.cu, replay_lpt16.cu): predicated cp.async / st.shared,
+// clamped shifts and 64-bit mask bit operations.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace convgpu {
+namespace lpt {
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)), "l"(src) : "memory");
+}
+// predicated forms (one predicated instruction, no divergent branch)
+__device__ __forceinline__ void cp_async4_if(uint32_t* dst, const uint32_t* src, bool on) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q cp.async.ca.shared.global [%0], [%1], 4; }"
+               ::"r"(smem_addr(dst)), "l"(src), "r"((uint32_t)on) : "memory");
+}
+__device__ __forceinline__ void cp_wait0_if(bool on) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q cp.async.wait_group 0; }" ::"r"((uint32_t)on) : "memory");
+}
+__device__ __forceinline__ void sts_if(uint32_t* dst, uint32_t v, bool on) {  // predicated st.shared
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q st.shared.u32 [%0], %1; }"
+               ::"r"(smem_addr(dst)), "r"(v), "r"((uint32_t)on) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
+// PTX shifts clamp: a shift by >= 32 gives 0 (no guard instructions, unlike
+// C++ where it is undefined); b - 32 wraps to a huge count for b < 32.
+__device__ __forceinline__ uint32_t shl_c(uint32_t v, uint32_t s) {
+  uint32_t r;
+  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
+  return r;
+}
+__device__ __forceinline__ uint32_t shr_c(uint32_t v, uint32_t s) {
+  uint32_t r;
+  asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
+  return r;
+}
+__device__ __forceinline__ bool bit64(uint32_t lo, uint32_t hi, uint32_t b) {  // b < 64
+  return ((shr_c(lo, b) | shr_c(hi, b - 32u)) & 1u) != 0;
+}
+__device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bool on) {  // b < 64
+  const uint32_t ml = shl_c(1u, b), mh = shl_c(1u, b - 32u);
+  lo = on ? (lo | ml) : (lo & ~ml);
+  hi = on ? (hi | mh) : (hi & ~mh);
+}
+__device__ __forceinline__ uint32_t ffs64(uint32_t lo, uint32_t hi) {  // lowest set bit, 64 if none
+  const uint32_t a = (uint32_t)__ffs(lo), b = (uint32_t)__ffs(hi);  // both always: no branch
+  return a ? a - 1u : (b ? b + 31u : 64u);
+}
+__device__ __forceinline__ uint32_t fls64(uint32_t lo, uint32_t hi) {  // highest set bit
+  return hi ? 63u - (uint32_t)__clz(hi) : 31u - (uint32_t)__clz(lo);
+}
+__device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi) {  // bits < r
+  lo = r >= 32 ? 0xFFFFFFFFu : ((1u << r) - 1u);
+  hi = r >= 64 ? 0xFFFFFFFFu : (r <= 32 ? 0u : ((1u << (r - 32)) - 1u));
+}
+
+}  // namespace lpt
+}  // namespace convgpu

@@ -33,6 +33,7 @@
 
 #include "common.cuh"
 #include "internal.h"
+#include "lpt_util.cuh"
 
 namespace convgpu {
 namespace lpt {
@@ -66,60 +67,6 @@ __host__ __device__ inline size_t warp_bytes(int policy, uint32_t n) {
   size_t b = (size_t)(W_BASE_WORDS + extra_words(policy)) * n * 32 * 4;
   if (policy == CONVGPU_RECENT_FIT) b += kStack * 32;
   return b;
-}
-
-__device__ __forceinline__ uint32_t smem_addr(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)), "l"(src) : "memory");
-}
-// predicated forms (one predicated instruction, no divergent branch)
-__device__ __forceinline__ void cp_async4_if(uint32_t* dst, const uint32_t* src, bool on) {
-  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q cp.async.ca.shared.global [%0], [%1], 4; }"
-               ::"r"(smem_addr(dst)), "l"(src), "r"((uint32_t)on) : "memory");
-}
-__device__ __forceinline__ void cp_wait0_if(bool on) {
-  asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q cp.async.wait_group 0; }" ::"r"((uint32_t)on) : "memory");
-}
-__device__ __forceinline__ void sts_if(uint32_t* dst, uint32_t v, bool on) {  // predicated st.shared
-  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q st.shared.u32 [%0], %1; }"
-               ::"r"(smem_addr(dst)), "r"(v), "r"((uint32_t)on) : "memory");
-}
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
-__device__ __forceinline__ void cp_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
-
-// PTX shifts clamp: a shift by >= 32 gives 0 (no guard instructions, unlike
-// C++ where it is undefined); b - 32 wraps to a huge count for b < 32.
-__device__ __forceinline__ uint32_t shl_c(uint32_t v, uint32_t s) {
-  uint32_t r;
-  asm("shl.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
-  return r;
-}
-__device__ __forceinline__ uint32_t shr_c(uint32_t v, uint32_t s) {
-  uint32_t r;
-  asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
-  return r;
-}
-__device__ __forceinline__ bool bit64(uint32_t lo, uint32_t hi, uint32_t b) {  // b < 64
-  return ((shr_c(lo, b) | shr_c(hi, b - 32u)) & 1u) != 0;
-}
-__device__ __forceinline__ void set64(uint32_t& lo, uint32_t& hi, uint32_t b, bool on) {  // b < 64
-  const uint32_t ml = shl_c(1u, b), mh = shl_c(1u, b - 32u);
-  lo = on ? (lo | ml) : (lo & ~ml);
-  hi = on ? (hi | mh) : (hi & ~mh);
-}
-__device__ __forceinline__ uint32_t ffs64(uint32_t lo, uint32_t hi) {  // lowest set bit, 64 if none
-  const uint32_t a = (uint32_t)__ffs(lo), b = (uint32_t)__ffs(hi);  // both always: no branch
-  return a ? a - 1u : (b ? b + 31u : 64u);
-}
-__device__ __forceinline__ uint32_t fls64(uint32_t lo, uint32_t hi) {  // highest set bit
-  return hi ? 63u - (uint32_t)__clz(hi) : 31u - (uint32_t)__clz(lo);
-}
-__device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi) {  // bits < r
-  lo = r >= 32 ? 0xFFFFFFFFu : ((1u << r) - 1u);
-  hi = r >= 64 ? 0xFFFFFFFFu : (r <= 32 ? 0u : ((1u << (r - 32)) - 1u));
 }
 
 // NF, KF: compile-time container / op counts (64, 4 for the configs) or 0.
@@ -417,6 +364,25 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     }
   };
 
+  // only_marked: the traces replay_lpt16.cu left to this kernel (8 markers
+  // probed per step, all loads in flight)
+  auto next = [&](uint64_t j) -> uint64_t {
+    if (!p.only_marked) return j;
+    while (j < p.count) {
+      uint32_t m[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint64_t jj = j + (uint64_t)u * T;
+        m[u] = jj < p.count ? p.admit_tick[jj * n] : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (m[u] == kLpt16Mark) return j + (uint64_t)u * T;
+      j += 8 * T;
+    }
+    return j;
+  };
+  i = next(i);
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
   if (have) { init(i); tdone = flags != 0; dmode = false; }  // static flags: no events
@@ -652,7 +618,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
     } while (!__all_sync(kFull, !have || tdone));
     if (have) {
       epilogue(i);
-      i += T;
+      i = next(i + T);
       have = i < p.count;
       if (have) { init(i); tdone = flags != 0; dmode = false; }
     }
@@ -708,6 +674,7 @@ static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
       cudaSuccess)
     return e;
   if (per_sm < 1) return cudaErrorInvalidConfiguration;
+  if (a.per_sm_cap && (uint32_t)per_sm > a.per_sm_cap) per_sm = (int)a.per_sm_cap;
   const uint64_t need = (a.count + threads - 1) / threads;
   uint64_t grid = (uint64_t)sms * (uint64_t)per_sm;
   if (a.grid_override) grid = a.grid_override;

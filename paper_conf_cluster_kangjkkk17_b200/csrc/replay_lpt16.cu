@@ -1,0 +1,616 @@
+// replay_lpt16.cu — lane-per-trace replay of ConVGPU's GPU-memory scheduler
+// (§III-D, Fig. 3) with COMPACT per-container
+// state, so that two warps per scheduler (8 per SM) fit in shared memory.
+//
+// Same algorithm and the same branch-free micro-step structure as
+// replay_lpt.cu; what differs is the state layout:
+//  * 14 bytes per container instead of 24 (n = 64: 896 B per trace, 28 KB per
+//    warp): key (u32), ust (u32: used 16 | op index 3 | FIRST | PAUSED |
+//    ADMITTED | op kinds 2 x K), sd (u32: size of the current op, saturated
+//    to 16 bits | delta of the next op 16), L (u16);
+//  * no admission word: an admission is stored straight to admit_tick (as
+//    tick << 6 | rank) and read back by the epilogue; the finish tick lives
+//    in the container's key after FINISH (0x80000000 | tick) and a paused
+//    container's key is 0xC0000000 (Recent-Fit: | the next container down the
+//    suspension stack, which is thereby a linked list needing no extra
+//    memory), both above every event key (ticks < 2^25 here);
+//  * Best-Fit keeps two bytes per container (rank of (L, index), container of
+//    rank) and the "same limit as the previous rank" bits in two registers;
+//  * the one-op-ahead fetch (raw op word + next delta, cp.async) lands in a
+//    2-word staging slot and is packed into the container's sd word at the
+//    end of the NEXT iteration, so the copy has a whole iteration to land
+//    (a register destination would make the compiler wait for it at the loop
+//    head); an event of the container fetched in the previous iteration
+//    (rare) takes a warp-uniform slow path.
+// A trace qualifies when every limit is <= 0xFFFE MiB, every delta <= 0xFFFF
+// ticks and its horizon (R19) < 2^25 (BASELINE configs [1]-[4] all do; the
+// 16-bit fields are then exact: a saturated size is above every limit, so it
+// is rejected / flagged exactly as the full size would be).  Other traces are
+// marked (admit_tick[trace][0] = kMark) and replayed by the 32-bit
+// lane-per-trace kernel in a second launch that skips unmarked traces.
+// Semantics are identical to replay_lpt.cu / replay.cu; every
+// GPU parity test runs this kernel against the oracle too.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "common.cuh"
+#include "internal.h"
+#include "lpt_util.cuh"
+
+namespace convgpu {
+namespace lpt16 {
+
+using lpt::ffs64;
+using lpt::fls64;
+using lpt::lowmask64;
+using lpt::shl_c;
+using lpt::sts_if;
+
+constexpr uint32_t N = 64, KOPS = 4;  // compile-time shape (configs [2]-[4])
+// ust word
+constexpr uint32_t kUsedMask = 0xFFFFu;
+constexpr uint32_t kKShift = 16;
+constexpr uint32_t kKOne = 1u << kKShift;
+constexpr uint32_t kFirst = 1u << 19;
+constexpr uint32_t kPaused = 1u << 20;
+constexpr uint32_t kAdmitted = 1u << 21;
+constexpr uint32_t kNotArrived = kPaused | kAdmitted;
+constexpr uint32_t kKindShift = 22;
+constexpr uint32_t kKindsMask = 0xFFu << kKindShift;
+// keys
+constexpr uint32_t kDone = 0x80000000u;    // | finish tick
+constexpr uint32_t kPausedKey = 0xC0000000u;  // | suspension number
+constexpr uint32_t kNoC = 64u;
+constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
+constexpr uint32_t kCompactHorizon = 1u << 25;
+constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
+
+// bytes per lane (= per trace) and warps per CTA (one CTA per SM)
+__host__ __device__ constexpr uint32_t extra_bytes(int policy) {
+  return policy == CONVGPU_BEST_FIT ? N * 2u : 0u;  // Best-Fit: rank_of / pi bytes
+}
+__host__ __device__ constexpr uint32_t lane_bytes(int policy) {
+  return N * 14u + extra_bytes(policy) + 8u;  // + 2-word fetch staging slot
+}
+__host__ __device__ constexpr int warps_per_cta(int policy) {
+  return policy == CONVGPU_BEST_FIT ? 7 : 8;
+}
+
+__device__ __forceinline__ uint32_t comp(const uint4& v, int j) {
+  return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
+}
+__device__ __forceinline__ void stg_if(uint32_t* p, uint32_t v, bool on) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q st.global.u32 [%0], %1; }"
+               ::"l"(p), "r"(v), "r"((uint32_t)on) : "memory");
+}
+__device__ __forceinline__ uint32_t pack_sd(uint32_t cw, uint32_t d) {
+  return min(cw & kSizeMask, 0xFFFFu) | (d << 16);
+}
+
+template <int POLICY>
+__global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_kernel(const ReplayArgs p) {
+  extern __shared__ __align__(16) uint32_t smem_w[];
+  const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+  constexpr uint32_t n = N, K = KOPS;
+  const uint32_t cap = p.cap, ovh = p.ovh;
+  uint32_t* const W0 = smem_w + wib * (32u * lane_bytes(POLICY) / 4u);
+  // word w of container c of this lane at W0[(w*n + c)*32 + lane]; limits as
+  // u16 pairs (containers 2j, 2j+1 in word j); then the policy's extra state
+  uint32_t* const s_key = W0 + lane;
+  uint32_t* const s_ust = W0 + 1 * n * 32 + lane;
+  uint32_t* const s_sd = W0 + 2 * n * 32 + lane;
+  uint32_t* const s_Lw = W0 + 3 * n * 32 + lane;
+  uint16_t* const s_L = reinterpret_cast<uint16_t*>(s_Lw);
+  // Best-Fit: rank of container c in (L, index) order and container of rank
+  // r, bytes (byte e of this lane at [(e >> 2) * 128 + (e & 3)])
+  uint8_t* const s_rof = reinterpret_cast<uint8_t*>(W0 + (3 * n + n / 2) * 32) + lane * 4;
+  uint8_t* const s_pi = reinterpret_cast<uint8_t*>(W0 + (3 * n + n / 2 + n / 4) * 32) + lane * 4;
+  // staging slot of the one-op-ahead fetch: {op word, delta of the op after}
+  uint32_t* const s_stg = W0 + (3 * n + n / 2 + extra_bytes(POLICY) / 4) * 32 + lane;
+#define AT(arr, c) (arr)[(c) * 32u]
+#define LIM(c) s_L[((c) >> 1) * 64u + ((c) & 1u)]
+#define ROF(c) s_rof[((c) >> 2) * 128u + ((c) & 3u)]
+#define PI(r) s_pi[((r) >> 2) * 128u + ((r) & 3u)]
+
+  const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+
+  unsigned long long st_traces = 0, st_events = 0, st_mk = 0, st_wait = 0, st_rej = 0,
+                     st_sel = 0, st_dig = 0;
+  uint32_t st_maxmk = 0, st_maxpk = 0;
+  unsigned long long racc_r = ~0ull, racc = 0;
+
+  uint32_t gmin[8];
+  uint32_t piv[8];
+  uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, rank = 0, draws = 0,
+           n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
+  uint32_t pm_lo = 0, pm_hi = 0, pr_lo = 0, pr_hi = 0;
+  uint32_t eq_lo = 0, eq_hi = 0;  // Best-Fit: rank r has the same limit as rank r - 1
+  uint32_t ru_head = kNoC;        // Recent-Fit: top of the suspension stack (linked
+                                  // through the paused containers' keys)
+  // the op fetched in the previous iteration: container, op word, delta
+  uint32_t pre_c = kNoC;
+  bool skip = false;
+#ifdef LPT16_DEBUG
+  uint32_t dbg0 = 0, dbg1 = 0, dbg2 = 0, dbg3 = 0, dbg4 = 0;
+#endif
+  const uint32_t* trace_delta = nullptr;
+  const uint32_t* trace_arg = nullptr;
+  uint32_t* adm_out = nullptr;
+
+  auto regroup = [&](uint32_t c) {
+    const uint32_t g = c >> 3, b = g << 3;
+    uint32_t v[8];
+#pragma unroll
+    for (uint32_t j = 0; j < 8; ++j) v[j] = AT(s_key, b + j);
+    const uint32_t m =
+        min(min(min(v[0], v[1]), min(v[2], v[3])), min(min(v[4], v[5]), min(v[6], v[7])));
+#pragma unroll
+    for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? m : gmin[j];
+  };
+
+  auto init = [&](uint64_t ti) {
+    const uint4* A4 = reinterpret_cast<const uint4*>(p.arrival + ti * n);
+    const uint4* L4 = reinterpret_cast<const uint4*>(p.limit + ti * n);
+    trace_delta = p.delta + ti * (uint64_t)K * n;
+    trace_arg = p.arg + ti * (uint64_t)K * n;
+    adm_out = p.admit_tick + ti * n;
+    const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
+    const uint4* R4 = reinterpret_cast<const uint4*>(trace_arg);
+    uint32_t bad = 0, lsum = 0, amax = 0, prev = 0, lmax = 0, dmax = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) gmin[j] = kKeyNone;
+#pragma unroll
+    for (uint32_t q = 0; q < 16; ++q) {
+      const uint4 a4 = __ldg(A4 + q), l4 = __ldg(L4 + q);
+      uint4 d4[4], w4[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) { d4[k] = __ldg(D4 + k * 16 + q); w4[k] = __ldg(R4 + k * 16 + q); }
+      uint32_t lp[2] = {0, 0};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t c = 4 * q + j, a = comp(a4, j), L = comp(l4, j);
+        if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+        if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
+        prev = a;
+        amax = max(amax, a);
+        lmax = max(lmax, L);
+        uint32_t kinds = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const uint32_t d = comp(d4[k], j), w = comp(w4[k], j);
+          lsum = min(lsum + min(d, kTickLimit), kTickLimit);
+          dmax = max(dmax, d);
+          if (((w >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+          kinds |= (w >> 30) << (2 * k);
+        }
+        const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
+        AT(s_key, c) = key;
+        AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu);
+        AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
+        lp[j >> 1] |= min(L, 0xFFFFu) << (16 * (j & 1));
+        gmin[c >> 3] = min(gmin[c >> 3], key);
+      }
+      s_Lw[(2 * q) * 32] = lp[0];
+      s_Lw[(2 * q + 1) * 32] = lp[1];
+    }
+    if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
+    // not representable in the 16-bit fields: the 32-bit kernel replays it
+    skip = bad == 0 && (lmax > 0xFFFEu || dmax > 0xFFFFu || amax + lsum >= kCompactHorizon);
+    if (skip) adm_out[0] = kLpt16Mark;
+    if (POLICY == CONVGPU_BEST_FIT) {
+      uint32_t v[64];
+#pragma unroll
+      for (int c = 0; c < 64; ++c) v[c] = ((uint32_t)LIM(c) << 6) | (uint32_t)c;
+#pragma unroll
+      for (int k = 2; k <= 64; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+#pragma unroll
+          for (int x = 0; x < 64; ++x) {
+            const int y = x ^ j;
+            if (y > x) {
+              const uint32_t a = v[x], b = v[y];
+              const bool up = (x & k) == 0;
+              v[x] = up ? min(a, b) : max(a, b);
+              v[y] = up ? max(a, b) : min(a, b);
+            }
+          }
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) piv[j] = v[8 * j + 7] >> 6;
+      uint32_t prevL = 0xFFFFFFFFu;
+      eq_lo = eq_hi = 0;
+#pragma unroll
+      for (int r = 0; r < 64; ++r) {
+        const uint32_t c = v[r] & 63u, Lc = v[r] >> 6;
+        if (Lc == prevL) { if (r < 32) eq_lo |= 1u << r; else eq_hi |= 1u << (r - 32); }
+        prevL = Lc;
+        ROF(c) = (uint8_t)r;
+        PI(r) = (uint8_t)c;
+      }
+    }
+    flags = bad;
+    free_mem = cap; target = kNoC; a_tg = 0; used_total = 0; rank = 0; draws = 0;
+    n_rej = 0; n_sel = 0; peak_res = 0; peak_used = 0; live = n; events = 0;
+    pm_lo = pm_hi = pr_lo = pr_hi = 0;
+    pre_c = kNoC;
+    ru_head = kNoC;
+  };
+
+  auto epilogue = [&](uint64_t ti) {
+    lpt::cp_wait0();
+    const bool stopped = (flags & kStopMask) != 0;
+    if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
+    const uint32_t* A = p.arrival + ti * n;
+    uint64_t dig = 0, swait = 0;
+    uint32_t mfin = 0;
+    const uint64_t ob = ti * n;
+    const uint4* A4 = reinterpret_cast<const uint4*>(A);
+    const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
+    const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
+#pragma unroll 4
+    for (uint32_t q = 0; q < 16; ++q) {
+      uint4 a4 = make_uint4(0, 0, 0, 0), m4 = a4, d4[4];
+      if (!stopped) {
+        a4 = __ldg(A4 + q);
+        m4 = M4[q];  // admissions this thread stored during the replay (coherent load)
+#pragma unroll
+        for (int k = 0; k < 4; ++k) d4[k] = __ldg(D4 + k * 16 + q);
+      }
+      uint32_t at[4], ar[4], wt[4], fn[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t c = 4 * q + j;
+        at[j] = kKeyNone; ar[j] = 0xFFu; wt[j] = 0; fn[j] = 0;
+        if (!stopped) {
+          if (AT(s_ust, c) & kAdmitted) {
+            const uint32_t adm = comp(m4, j);
+            at[j] = adm >> 6;
+            ar[j] = adm & 63u;
+          }
+          fn[j] = AT(s_key, c) & ~kDone;
+          // R17: wait = finish - arrival - sum of deltas
+          wt[j] = fn[j] - comp(a4, j) - comp(d4[0], j) - comp(d4[1], j) - comp(d4[2], j) -
+                  comp(d4[3], j);
+        }
+        const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
+        dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
+        mfin = max(mfin, fn[j]);
+        swait += wt[j];
+      }
+      // streaming stores (evict-first): outputs are not re-read, inputs of the
+      // traces in flight should stay in L2
+      __stcs(reinterpret_cast<uint4*>(p.admit_tick + ob) + q, make_uint4(at[0], at[1], at[2], at[3]));
+      if (p.admit_rank)
+        __stcs(reinterpret_cast<unsigned int*>(p.admit_rank + ob) + q,
+               ar[0] | (ar[1] << 8) | (ar[2] << 16) | (ar[3] << 24));
+      if (p.wait) __stcs(reinterpret_cast<uint4*>(p.wait + ob) + q, make_uint4(wt[0], wt[1], wt[2], wt[3]));
+      if (p.finish) __stcs(reinterpret_cast<uint4*>(p.finish + ob) + q, make_uint4(fn[0], fn[1], fn[2], fn[3]));
+    }
+    const uint32_t makespan = stopped ? 0u : mfin - __ldg(A);
+    dig += mix64(((uint64_t)makespan << 32) | peak_res);
+    dig += mix64(((uint64_t)peak_used << 32) | flags);
+    dig += mix64(swait);
+    dig += mix64(((uint64_t)n_rej << 32) | n_sel);
+    if (p.summary) {
+      convgpu_summary_t sm;
+      sm.makespan = makespan; sm.peak_reserved = peak_res; sm.peak_used = peak_used;
+      sm.flags = flags; sm.sum_wait = swait; sm.n_rejected = n_rej; sm.n_select = n_sel;
+      sm.digest = dig;
+#ifdef LPT16_DEBUG
+      if (flags & CONVGPU_FLAG_INVALID_FREE) {
+        sm.makespan = dbg0; sm.peak_reserved = dbg1; sm.peak_used = dbg2; sm.n_rejected = dbg3;
+        sm.n_select = dbg4; sm.sum_wait = events;
+      }
+#endif
+      p.summary[ti] = sm;
+    }
+    st_traces += 1; st_events += events; st_mk += makespan; st_wait += swait; st_rej += n_rej;
+    st_sel += n_sel; st_dig += dig;
+    st_maxmk = max(st_maxmk, makespan);
+    st_maxpk = max(st_maxpk, peak_res);
+    if (flags && p.stats)
+      for (int b = 0; b < 8; ++b)
+        if ((flags >> b) & 1u) atomicAdd(&p.stats->flag_count[b], 1u);
+    if (p.range_digest) {
+      const unsigned long long r = (p.tid_base + ti) / p.range_size;
+      if (r != racc_r) {
+        if (racc_r != ~0ull) atomicAdd((unsigned long long*)&p.range_digest[racc_r], racc);
+        racc_r = r;
+        racc = 0;
+      }
+      racc += dig;
+    }
+  };
+
+  bool have = i < p.count, tdone = false, dmode = false;
+  uint32_t cur_t = 0;
+  if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
+  while (__any_sync(kFull, have)) {
+    do {
+      if (have && !tdone) {
+        uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
+        if (!dmode) {
+          // ================= EVENT step (a2 + a3), branch-free =================
+          const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
+          const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
+          const uint32_t kmin = min(min(m01, m23), min(m45, m67));
+          if (kmin >= kDone) {
+            if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
+            tdone = true;
+          } else {
+            const uint32_t t = kmin >> 6, c = kmin & 63u;
+            cur_t = t;
+            ++events;
+            // the container fetched in the previous iteration: its op data are
+            // still in registers (rare: warp-uniform slow path)
+            if (__any_sync(__activemask(), c == pre_c)) {
+              if (c == pre_c) {
+                lpt::cp_wait0();
+                AT(s_sd, c) = pack_sd(AT(s_stg, 0), AT(s_stg, 1));
+                pre_c = kNoC;
+              }
+            }
+            const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
+            const bool arr = (ust & kNotArrived) == kNotArrived;
+            const uint32_t k = (ust >> kKShift) & 7u;
+            const uint32_t kind = (ust >> (kKindShift + 2 * k)) & 3u;
+            const uint32_t r = sd & 0xFFFFu, used = ust & kUsedMask;
+            const uint32_t nd = arr ? used : (sd >> 16);  // d_0 before arrival
+            const bool isA = !arr && kind == CONVGPU_OP_ALLOC;
+            const bool isF = !arr && kind == CONVGPU_OP_FREE;
+            const bool isX = !arr && kind == CONVGPU_OP_FINISH;
+            const bool tnone = target == kNoC, ctg = c == target;
+            const uint32_t a_c = (ust & kAdmitted) ? L : (ctg ? a_tg : 0u);
+            // ARRIVE (Fig. 3b/3c; R2)
+            const uint32_t g = (arr && tnone) ? min(L, free_mem) : 0u;
+            const bool vadm = arr && g == L;
+            const bool vtgt = arr && !vadm && g > 0;
+            // ALLOC
+            const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
+            const bool rej = isA && need > L;                // R10
+            const bool grant = isA && !rej && need <= a_c;
+            const bool pause = isA && !rej && !grant;       // reply withheld
+            // FREE (R11)
+            const bool badfree = isF && r > used;
+            free_mem = free_mem - g + (isX ? a_c : 0u);
+            used_total = used_total + (grant ? need - used : 0u) - ((isF && !badfree) ? r : 0u) -
+                         (isX ? used : 0u);
+            peak_res = max(peak_res, cap - free_mem);
+            peak_used = max(peak_used, used_total);
+            if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+            const bool clear_tg = isX && ctg;               // R20
+            target = vtgt ? c : (clear_tg ? kNoC : target);
+            a_tg = vtgt ? g : (clear_tg ? 0u : a_tg);
+            stg_if(adm_out + c, (t << 6) | rank, vadm);     // admission at arrival
+            rank += vadm ? 1u : 0u;
+            n_rej += rej ? 1u : 0u;
+            live -= isX ? 1u : 0u;
+            const uint32_t pmask = pause ? 0xFFFFFFFFu : 0u;
+            pm_lo |= shl_c(1u, c) & pmask;
+            pm_hi |= shl_c(1u, c - 32u) & pmask;
+            if (POLICY == CONVGPU_BEST_FIT) {
+              const uint32_t rc = ROF(c);
+              pr_lo |= shl_c(1u, rc) & pmask;
+              pr_hi |= shl_c(1u, rc - 32u) & pmask;
+            }
+            // Recent-Fit: push c on the suspension stack (its key links the old
+            // top) unless it is the fill target, which resumes without a
+            // selection (R1) and so must never be popped
+            const uint32_t plink = (POLICY == CONVGPU_RECENT_FIT) ? ru_head : 0u;
+            if (POLICY == CONVGPU_RECENT_FIT) ru_head = (pause && !ctg) ? c : ru_head;
+            dmode = (pause & tnone) | (isX & ((target != kNoC) | ((pm_lo | pm_hi) != 0u)));
+            if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true;
+#ifdef LPT16_DEBUG
+              dbg0 = c | (k << 8) | ((uint32_t)(pre_c) << 16); dbg1 = r; dbg2 = used; dbg3 = ust; dbg4 = sd;
+#endif
+            }
+            const bool adv = !isX && !pause && !badfree;
+            uint32_t nu = ust;
+            nu = grant ? ((ust & ~kUsedMask) | need | kFirst) : nu;
+            nu = (isF && !badfree) ? ust - r : nu;
+            nu = isX ? (ust & ~kUsedMask) : nu;
+            nu = pause ? (ust | kPaused) : nu;
+            nu = arr ? ((vadm ? kAdmitted : 0u) | (ust & kKindsMask)) : nu;
+            nu = (adv && !arr) ? nu + kKOne : nu;
+            AT(s_ust, c) = nu;
+            kc = badfree ? kNoC : c;
+            nkc = adv ? (((t + nd) << 6) | c) : (isX ? (kDone | t) : (kPausedKey | plink));
+            pfk = (adv && !arr) ? k + 1u : 0xFFu;
+          }
+        } else {
+          // ====== one DISPATCH step at the triggering tick (R1, R9) ======
+          const uint32_t t = cur_t;
+          if (POLICY == CONVGPU_FIFO) {
+            const bool ns = target == kNoC;
+            const uint32_t sel = ffs64(pm_lo, pm_hi);
+            target = ns ? sel : target;
+            a_tg = ns ? 0u : a_tg;
+            n_sel += ns ? 1u : 0u;
+          } else if (target == kNoC) {
+            uint32_t sel;
+            if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4
+              uint32_t gc = 0;
+#pragma unroll
+              for (int j = 0; j < 8; ++j) gc += (piv[j] <= free_mem) ? 1u : 0u;
+              const uint32_t rb = min(gc, 7u) * 8u;
+              uint32_t in = 0;
+#pragma unroll
+              for (uint32_t j = 0; j < 8; ++j) in += ((uint32_t)LIM(PI(rb + j)) <= free_mem) ? 1u : 0u;
+              const uint32_t lo = (gc == 8u) ? 64u : rb + in;
+              uint32_t ml, mh;
+              lowmask64(lo, ml, mh);
+              const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
+              const uint32_t h = min(fls64(fl, fh), n - 1u);
+              // first rank of h's limit group: the highest rank <= h that
+              // starts a group (rank 0 always does)
+              uint32_t hl, hh, gl, gh;
+              lowmask64(h + 1u, hl, hh);
+              lowmask64(fls64(~eq_lo & hl, ~eq_hi & hh), gl, gh);
+              const uint32_t r_fit = ffs64(pr_lo & ~gl, pr_hi & ~gh);
+              const uint32_t r_min = ffs64(pr_lo, pr_hi);
+              sel = PI((fl | fh) ? r_fit : r_min);
+            } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
+              // pop the suspension stack: paused containers leave the paused
+              // set only by resuming, and only the target resumes, so popping
+              // at selection keeps the stack exactly the paused set in
+              // suspension order
+              sel = ru_head;
+              ru_head = AT(s_key, sel) & 127u;
+            } else {  // RANDOM_FIT (R6)
+              const uint64_t tid = p.tid_base + i;
+              const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
+              const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                         (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+              ++draws;
+              const uint32_t jj = __umulhi(x.x, m);
+              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+            }
+            target = sel;
+            a_tg = 0;
+            ++n_sel;
+          }
+          {
+            // the target was not fetched in the previous iteration: a dispatch
+            // step follows a pause / FINISH (no fetch) or an admission, after
+            // which the resumed container is no longer paused
+            const uint32_t tg = target;
+            const uint32_t Lt = LIM(tg), ut = AT(s_ust, tg), sdt = AT(s_sd, tg);
+            const uint32_t g = min(free_mem, Lt - a_tg);
+            a_tg += g;
+            free_mem -= g;
+            const uint32_t pend = (sdt & 0xFFFFu) + ((ut & kFirst) ? 0u : ovh);
+            const uint32_t uu = ut & kUsedMask;
+            const bool res = (ut & kPaused) && uu + pend <= a_tg;  // RESUME (R9)
+            const bool full = a_tg == Lt;                          // admit, cascade
+            used_total += res ? pend : 0u;
+            peak_res = max(peak_res, cap - free_mem);
+            peak_used = max(peak_used, used_total);
+            if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
+            uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
+            nu |= full ? kAdmitted : 0u;
+            AT(s_ust, tg) = nu;
+            const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;
+            pm_lo &= ~(shl_c(1u, tg) & rmask);
+            pm_hi &= ~(shl_c(1u, tg - 32u) & rmask);
+            if (POLICY == CONVGPU_BEST_FIT) {
+              const uint32_t rt = ROF(tg);
+              pr_lo &= ~(shl_c(1u, rt) & rmask);
+              pr_hi &= ~(shl_c(1u, rt - 32u) & rmask);
+            }
+            stg_if(adm_out + tg, (t << 6) | rank, full);
+            rank += full ? 1u : 0u;
+            target = full ? kNoC : target;
+            a_tg = full ? 0u : a_tg;
+            dmode = full && (pm_lo | pm_hi) != 0u;
+            kc = res ? tg : kNoC;
+            nkc = ((t + (sdt >> 16)) << 6) | tg;
+            pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
+          }
+        }
+        // ---- shared tail: key update, group re-min, retire the previous
+        // iteration's fetch, issue this iteration's ----
+        {
+          const uint32_t kcs = kc & 63u;
+          sts_if(&AT(s_key, kcs), nkc, kc != kNoC);
+          regroup(kcs);
+          // retire last iteration's fetch (issued one iteration ago)
+          lpt::cp_wait0_if(pre_c != kNoC);
+          sts_if(&AT(s_sd, pre_c & 63u), pack_sd(AT(s_stg, 0), AT(s_stg, 1)), pre_c != kNoC);
+          // op k word and the delta of op k+1 (clamped: FINISH never reads it)
+          const bool f = pfk < K;
+          const uint32_t off = pfk * n + kcs;
+          lpt::cp_async4_if(&AT(s_stg, 0), trace_arg + off, f);
+          lpt::cp_async4_if(&AT(s_stg, 1), trace_delta + min(pfk + 1u, K - 1u) * n + kcs, f);
+          lpt::cp_commit();
+          pre_c = f ? kcs : kNoC;
+        }
+      }
+    } while (!__all_sync(kFull, !have || tdone));
+    if (have) {
+      if (!skip) epilogue(i);
+      i += T;
+      have = i < p.count;
+      if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
+    }
+  }
+#undef PI
+#undef ROF
+#undef LIM
+#undef AT
+
+  if (p.range_digest && racc_r != ~0ull)
+    atomicAdd((unsigned long long*)&p.range_digest[racc_r], racc);
+  if (p.stats) {
+    __syncwarp();
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      st_traces += __shfl_xor_sync(kFull, st_traces, o);
+      st_events += __shfl_xor_sync(kFull, st_events, o);
+      st_mk += __shfl_xor_sync(kFull, st_mk, o);
+      st_wait += __shfl_xor_sync(kFull, st_wait, o);
+      st_rej += __shfl_xor_sync(kFull, st_rej, o);
+      st_sel += __shfl_xor_sync(kFull, st_sel, o);
+      st_dig += __shfl_xor_sync(kFull, st_dig, o);
+      st_maxmk = max(st_maxmk, __shfl_xor_sync(kFull, st_maxmk, o));
+      st_maxpk = max(st_maxpk, __shfl_xor_sync(kFull, st_maxpk, o));
+    }
+    if (lane == 0 && st_traces) {
+      convgpu_stats_t* Sg = p.stats;
+      atomicAdd((unsigned long long*)&Sg->traces, st_traces);
+      atomicAdd((unsigned long long*)&Sg->events, st_events);
+      atomicAdd((unsigned long long*)&Sg->sum_makespan, st_mk);
+      atomicAdd((unsigned long long*)&Sg->sum_wait, st_wait);
+      atomicAdd((unsigned long long*)&Sg->n_rejected, st_rej);
+      atomicAdd((unsigned long long*)&Sg->n_select, st_sel);
+      atomicAdd((unsigned long long*)&Sg->digest_sum, st_dig);
+      atomicMax(&Sg->max_makespan, st_maxmk);
+      atomicMax(&Sg->max_peak_reserved, st_maxpk);
+    }
+  }
+}
+
+template <int POLICY>
+static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
+  const int threads = 32 * warps_per_cta(POLICY);
+  const size_t smem = (size_t)threads * lane_bytes(POLICY);
+  auto kern = replay_lpt16_kernel<POLICY>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  const uint64_t need = (a.count + threads - 1) / threads;
+  uint64_t grid = (uint64_t)sms;  // one CTA per SM, persistent
+  if (a.grid_override) grid = a.grid_override;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  kern<<<(unsigned)grid, threads, smem, stream>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace lpt16
+
+bool lpt16_supported(const ReplayArgs& a) {
+  return a.n == lpt16::N && a.K == lpt16::KOPS && a.admit_tick != nullptr && a.aligned16;
+}
+
+cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream) {
+  cudaError_t e;
+  switch (policy) {
+    case CONVGPU_FIFO: e = lpt16::launch_t<CONVGPU_FIFO>(a, stream); break;
+    case CONVGPU_BEST_FIT: e = lpt16::launch_t<CONVGPU_BEST_FIT>(a, stream); break;
+    case CONVGPU_RECENT_FIT: e = lpt16::launch_t<CONVGPU_RECENT_FIT>(a, stream); break;
+    case CONVGPU_RANDOM_FIT: e = lpt16::launch_t<CONVGPU_RANDOM_FIT>(a, stream); break;
+    default: return cudaErrorInvalidValue;
+  }
+  if (e != cudaSuccess) return e;
+  // traces the 16-bit layout cannot hold: the 32-bit lane kernel, marked only
+  ReplayArgs b = a;
+  b.only_marked = 1;
+  return launch_replay_lpt(b, policy, stream);
+}
+
+}  // namespace convgpu

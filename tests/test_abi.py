@@ -42,8 +42,8 @@ def test_nm_lists_symbols_as_extern_c(so):
 
 
 def test_version_and_strerror(so):
-    assert so.convgpu_abi_version() == 2
-    assert so.convgpu_launches_per_call() == 1
+    assert so.convgpu_abi_version() == 3
+    assert so.convgpu_launches_per_call() == 2
     assert b"invalid" in so.convgpu_strerror(-errno.EINVAL)
     assert b"sm_100" in so.convgpu_strerror(-errno.ENODEV)
 
@@ -63,7 +63,8 @@ def _traces(**kw):
 
 @pytest.mark.parametrize("kw", [dict(n_containers=0), dict(n_containers=65), dict(n_ops=0),
                                 dict(n_ops=9), dict(arrival=None), dict(op_arg=None),
-                                dict(kernel_variant=3), dict(ctx_overhead_mib=1 << 30)])
+                                dict(kernel_variant=4), dict(ctx_overhead_mib=1 << 30),
+                                dict(kernel_variant=3, n_containers=16)])
 def test_replay_rejects_bad_shape_before_touching_the_device(so, kw):
     out = cg.OutT()
     assert so.convgpu_replay(C.byref(_traces(**kw)), 10, 1000, 0, C.byref(out)) == -errno.EINVAL

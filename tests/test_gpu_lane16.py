@@ -1,0 +1,137 @@
+"""GPU parity of the compact lane-per-trace kernel (csrc/replay_lpt16.cu,
+CONVGPU_KERNEL_LANE_COMPACT) against the C oracle, element by element, on
+every integer output: configs [2] and [4] (rho 8 has limits above the 16-bit
+fields, so its traces go through the marked 32-bit fallback launch), edge-case
+batches with tiny deltas (consecutive events of one container hit the
+register-fetch slow path), extreme values (fallback and static flags), a
+batch mixing eligible and ineligible traces, and the full-size config [2]
+sampled.  Needs a B200: run via gpurun."""
+import numpy as np
+import pytest
+
+import workloads as W
+from test_gpu_parity import POLS, _compare, _compare_stats, _extreme_batch, _gpu_replay
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def cg():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_cluster_kangjkkk17_b200 as m
+    from paper_conf_cluster_kangjkkk17_b200 import build
+    build.build()
+    return m
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_config2_window_ragged(cg, orc, policy):
+    w = W.CONFIGS["c2"]
+    base, N = 987_654_321_001, 4_741
+    ref = orc.replay_range(w, policy, base, base + N, full=True)
+    tr = cg.generate(w.gen, base, N)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+
+
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("rho", [1, 4, 7, 8])
+def test_lane16_rho_sweep(cg, orc, policy, rho):
+    w = W.rho_sweep(rho, rand_seed=rho * 7 + 1)
+    ref = orc.replay_range(w, policy, 10_000, 11_500, full=True)
+    tr = cg.generate(w.gen, 10_000, 1_500)
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+
+
+EDGE64 = [  # (cap, ovh, mode, count)
+    (256, 0, "valid", 700),
+    (512, 66, "valid", 500),
+    (300, 5, "mixed", 900),
+    (128, 0, "over", 500),
+    (200, 1, "delayed", 500),
+    (256, 0, "badfree", 400),
+]
+
+
+@pytest.mark.parametrize("case", EDGE64, ids=lambda c: f"{c[2]}{c[0]}o{c[1]}")
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_edge_batches(cg, orc, policy, case):
+    cap, ovh, mode, count = case
+    b = W.random_batch(4242 + cap, count, 64, 4, cap, ovh=ovh, mode=mode,
+                       limit_choices=range(0, cap + 1))
+    base = 7_000_000_000 + cap
+    ref = orc.replay_batch(b, cap, policy, tid_base=base, rand_seed=5 + cap, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=base)
+    out = _gpu_replay(cg, tr, cap, policy, seed=5 + cap, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_extreme_values_and_mixed_batch(cg, orc, policy):
+    """Values at the ABI limits (all ineligible or statically flagged),
+    interleaved with config-[2] traces that the compact kernel replays."""
+    xb, cap, ovh = _extreme_batch(95, 300, 64, 4)
+    ref = orc.replay_batch(xb, cap, policy, tid_base=2**63 + 5, rand_seed=2**64 - 1, ovh=ovh)
+    tr = cg.traces_from_numpy(xb.arrival, xb.limit, xb.delta, xb.arg, trace_id_base=2**63 + 5)
+    out = _gpu_replay(cg, tr, cap, policy, seed=2**64 - 1, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    # a mixed batch: small-valued traces (compact) next to large-valued ones (fallback)
+    sb = W.random_batch(96, 300, 64, 4, 16, ovh=1, mode="mixed", limit_choices=range(0, 17))
+    mix = W.Batch(64, 4, *(np.concatenate([getattr(sb, f), getattr(xb, f)])[np.argsort(
+        np.arange(600) % 7, kind="stable")] for f in ("arrival", "limit", "delta", "arg")))
+    ref = orc.replay_batch(mix, cap, policy, tid_base=11, rand_seed=3, ovh=ovh)
+    tr = cg.traces_from_numpy(mix.arrival, mix.limit, mix.delta, mix.arg, trace_id_base=11)
+    out = _gpu_replay(cg, tr, cap, policy, seed=3, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_full_size_sampled(cg, orc, policy):
+    """Config [2] at full size in the bench launch configuration (AUTO with full
+    outputs = the compact kernel): sampled traces against the oracle one by
+    one, stats and range digest against the outputs."""
+    w = W.CONFIGS["c2"]
+    N = w.n_traces
+    tr = cg.generate(w.gen, 0, N)
+    rs = 1 << 16
+    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, range_size=rs,
+                      range_count=(N + rs - 1) // rs)
+    s = out.summary_np()
+    full = out.full_np()
+    rng = np.random.default_rng(11)
+    idx = np.unique(np.concatenate([rng.integers(0, N, 200), [0, 1, N - 2, N - 1]]))
+    for i in idx:
+        ref = orc.replay_range(w, policy, int(i), int(i) + 1, full=True)
+        for f in ("makespan", "peak_reserved", "peak_used", "flags", "sum_wait", "n_rejected",
+                  "n_select", "digest"):
+            assert int(s[f][i]) == int(ref[f][0]), (i, f)
+        for f in ("admit_tick", "admit_rank", "wait", "finish"):
+            np.testing.assert_array_equal(full[f][i], ref[f][0], err_msg=f"{i} {f}")
+    st = cg.stats_dict(out.stats_np())
+    assert st["traces"] == N and st["events"] == N * w.events_per_trace()
+    assert st["flag_count"] == [0] * 8
+    assert st["digest_sum"] == int(s["digest"].astype(np.uint64).sum(dtype=np.uint64))
+    rd = out.range_digest.cpu().numpy().view(np.uint64)
+    assert int(rd.sum(dtype=np.uint64)) == st["digest_sum"]
+    ref = orc.replay_range(w, policy, 5 * rs, 6 * rs)
+    assert int(rd[5]) == int(ref["digest"].sum(dtype=np.uint64))
+
+
+def test_lane16_rejects_unsupported_shapes(cg):
+    w = W.CONFIGS["c1"]  # n = 16
+    tr = cg.generate(w.gen, 0, 64)
+    with pytest.raises(cg.ConvgpuError):
+        cg.replay(tr, w.cap, "fifo", cg.alloc_out(64, 16), kernel="lane16")
+    w2 = W.CONFIGS["c2"]
+    tr = cg.generate(w2.gen, 0, 64)
+    with pytest.raises(cg.ConvgpuError):  # admit_tick is the admission scratch
+        cg.replay(tr, w2.cap, "fifo", cg.alloc_out(64, 64, full=False), kernel="lane16")
+    with pytest.raises(cg.ConvgpuError):  # R1-LIT runs on the warp kernel only
+        cg.replay(tr, w2.cap, "fifo+literal", cg.alloc_out(64, 64), kernel="lane16")
