@@ -20,7 +20,8 @@ from typing import Optional
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_PKG, "libconvgpu.so")
+# CONVGPU_SO: an alternative build of the same library (A/B kernel tuning only)
+SO_PATH = os.environ.get("CONVGPU_SO") or os.path.join(_PKG, "libconvgpu.so")
 
 FIFO, BEST_FIT, RECENT_FIT, RANDOM_FIT = 0, 1, 2, 3
 LITERAL = 0x100  # CONVGPU_DISPATCH_LITERAL: OR into a policy for the R1-LIT reading

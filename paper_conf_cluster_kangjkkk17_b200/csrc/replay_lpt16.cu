@@ -121,6 +121,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   unsigned long long racc_r = ~0ull, racc = 0;
 
   uint32_t gmin[8];
+  // arrival + sum of deltas per container, in registers (R17's wait = finish -
+  // base is then computed without re-reading the trace in the epilogue)
+  constexpr bool kBaseRegs = POLICY != CONVGPU_BEST_FIT;  // Best-Fit: no register room
+  uint32_t base[kBaseRegs ? 64 : 1];
+  uint32_t arr0 = 0;
   uint32_t piv[8];
   uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, rank = 0, draws = 0,
            n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
@@ -175,10 +180,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         prev = a;
         amax = max(amax, a);
         lmax = max(lmax, L);
-        uint32_t kinds = 0;
+        uint32_t kinds = 0, bsum = a;
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
           const uint32_t d = comp(d4[k], j), w = comp(w4[k], j);
+          bsum += d;
           lsum = min(lsum + min(d, kTickLimit), kTickLimit);
           dmax = max(dmax, d);
           if (((w >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
@@ -190,6 +196,8 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
         lp[j >> 1] |= min(L, 0xFFFFu) << (16 * (j & 1));
         gmin[c >> 3] = min(gmin[c >> 3], key);
+        if (kBaseRegs) base[kBaseRegs ? c : 0] = bsum;
+        if (c == 0) arr0 = a;
       }
       s_Lw[(2 * q) * 32] = lp[0];
       s_Lw[(2 * q + 1) * 32] = lp[1];
@@ -250,14 +258,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     const uint4* A4 = reinterpret_cast<const uint4*>(A);
     const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
     const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
-#pragma unroll 4
+#pragma unroll(kBaseRegs ? 16 : 4)
     for (uint32_t q = 0; q < 16; ++q) {
-      uint4 a4 = make_uint4(0, 0, 0, 0), m4 = a4, d4[4];
+      uint4 a4 = make_uint4(0, 0, 0, 0), m4 = a4, d4[4] = {a4, a4, a4, a4};
       if (!stopped) {
-        a4 = __ldg(A4 + q);
         m4 = M4[q];  // admissions this thread stored during the replay (coherent load)
+        if (!kBaseRegs) {
+          a4 = __ldg(A4 + q);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) d4[k] = __ldg(D4 + k * 16 + q);
+          for (int k = 0; k < 4; ++k) d4[k] = __ldg(D4 + k * 16 + q);
+        }
       }
       uint32_t at[4], ar[4], wt[4], fn[4];
 #pragma unroll
@@ -272,8 +282,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           }
           fn[j] = AT(s_key, c) & ~kDone;
           // R17: wait = finish - arrival - sum of deltas
-          wt[j] = fn[j] - comp(a4, j) - comp(d4[0], j) - comp(d4[1], j) - comp(d4[2], j) -
-                  comp(d4[3], j);
+          wt[j] = kBaseRegs ? fn[j] - base[kBaseRegs ? c : 0]
+                            : fn[j] - comp(a4, j) - comp(d4[0], j) - comp(d4[1], j) -
+                                  comp(d4[2], j) - comp(d4[3], j);
         }
         const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
         dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
@@ -289,7 +300,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       if (p.wait) __stcs(reinterpret_cast<uint4*>(p.wait + ob) + q, make_uint4(wt[0], wt[1], wt[2], wt[3]));
       if (p.finish) __stcs(reinterpret_cast<uint4*>(p.finish + ob) + q, make_uint4(fn[0], fn[1], fn[2], fn[3]));
     }
-    const uint32_t makespan = stopped ? 0u : mfin - __ldg(A);
+    const uint32_t makespan = stopped ? 0u : mfin - arr0;
     dig += mix64(((uint64_t)makespan << 32) | peak_res);
     dig += mix64(((uint64_t)peak_used << 32) | flags);
     dig += mix64(swait);
@@ -346,14 +357,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             ++events;
             // the container fetched in the previous iteration: its op data are
             // still in registers (rare: warp-uniform slow path)
-            if (__any_sync(__activemask(), c == pre_c)) {
-              if (c == pre_c) {
-                lpt::cp_wait0();
-                AT(s_sd, c) = pack_sd(AT(s_stg, 0), AT(s_stg, 1));
-                pre_c = kNoC;
-              }
-            }
-            const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
+            // (predicated: wait, take the staged copy, store it, drop the retire)
+            const bool hz = c == pre_c;
+            lpt::cp_wait0_if(hz);
+            const uint32_t sdh = pack_sd(AT(s_stg, 0), AT(s_stg, 1));
+            sts_if(&AT(s_sd, c), sdh, hz);
+            const uint32_t ust = AT(s_ust, c), sdm = AT(s_sd, c), L = LIM(c);
+            const uint32_t sd = hz ? sdh : sdm;
+            pre_c = hz ? kNoC : pre_c;
             const bool arr = (ust & kNotArrived) == kNotArrived;
             const uint32_t k = (ust >> kKShift) & 7u;
             const uint32_t kind = (ust >> (kKindShift + 2 * k)) & 3u;
