@@ -123,8 +123,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   uint32_t gmin[8];
   // arrival + sum of deltas per container, in registers (R17's wait = finish -
   // base is then computed without re-reading the trace in the epilogue)
-  constexpr bool kBaseRegs = POLICY != CONVGPU_BEST_FIT;  // Best-Fit: no register room
-  uint32_t base[kBaseRegs ? 64 : 1];
+  uint32_t base[64];
   uint32_t arr0 = 0;
   uint32_t piv[8];
   uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, rank = 0, draws = 0,
@@ -196,7 +195,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
         lp[j >> 1] |= min(L, 0xFFFFu) << (16 * (j & 1));
         gmin[c >> 3] = min(gmin[c >> 3], key);
-        if (kBaseRegs) base[kBaseRegs ? c : 0] = bsum;
+        base[c] = bsum;
         if (c == 0) arr0 = a;
       }
       s_Lw[(2 * q) * 32] = lp[0];
@@ -251,24 +250,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     lpt::cp_wait0();
     const bool stopped = (flags & kStopMask) != 0;
     if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
-    const uint32_t* A = p.arrival + ti * n;
     uint64_t dig = 0, swait = 0;
     uint32_t mfin = 0;
     const uint64_t ob = ti * n;
-    const uint4* A4 = reinterpret_cast<const uint4*>(A);
-    const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
     const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
-#pragma unroll(kBaseRegs ? 16 : 4)
-    for (uint32_t q = 0; q < 16; ++q) {
-      uint4 a4 = make_uint4(0, 0, 0, 0), m4 = a4, d4[4] = {a4, a4, a4, a4};
-      if (!stopped) {
-        m4 = M4[q];  // admissions this thread stored during the replay (coherent load)
-        if (!kBaseRegs) {
-          a4 = __ldg(A4 + q);
 #pragma unroll
-          for (int k = 0; k < 4; ++k) d4[k] = __ldg(D4 + k * 16 + q);
-        }
-      }
+    for (uint32_t q = 0; q < 16; ++q) {
+      // admissions this thread stored during the replay (coherent load)
+      const uint4 m4 = stopped ? make_uint4(0, 0, 0, 0) : M4[q];
       uint32_t at[4], ar[4], wt[4], fn[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -282,9 +271,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           }
           fn[j] = AT(s_key, c) & ~kDone;
           // R17: wait = finish - arrival - sum of deltas
-          wt[j] = kBaseRegs ? fn[j] - base[kBaseRegs ? c : 0]
-                            : fn[j] - comp(a4, j) - comp(d4[0], j) - comp(d4[1], j) -
-                                  comp(d4[2], j) - comp(d4[3], j);
+          wt[j] = fn[j] - base[c];
         }
         const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
         dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
