@@ -36,6 +36,7 @@
 #include "common.cuh"
 #include "internal.h"
 #include "lpt_util.cuh"
+#include "oem64.cuh"
 
 namespace convgpu {
 namespace lpt16 {
@@ -209,22 +210,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       uint32_t v[64];
 #pragma unroll
       for (int c = 0; c < 64; ++c) v[c] = ((uint32_t)LIM(c) << 6) | (uint32_t)c;
-#pragma unroll
-      for (int k = 2; k <= 64; k <<= 1) {
-#pragma unroll
-        for (int j = k >> 1; j > 0; j >>= 1) {
-#pragma unroll
-          for (int x = 0; x < 64; ++x) {
-            const int y = x ^ j;
-            if (y > x) {
-              const uint32_t a = v[x], b = v[y];
-              const bool up = (x & k) == 0;
-              v[x] = up ? min(a, b) : max(a, b);
-              v[y] = up ? max(a, b) : min(a, b);
-            }
-          }
-        }
-      }
+      // Batcher's odd-even merge sort network (oem64.cuh): 543
+      // compare-exchanges for 64 keys, literal indices, v stays in registers
+#define OEM_CE(a, b) { const uint32_t x = v[a], y = v[b]; v[a] = min(x, y); v[b] = max(x, y); }
+      OEM64_NETWORK(OEM_CE)
+#undef OEM_CE
 #pragma unroll
       for (int j = 0; j < 8; ++j) piv[j] = v[8 * j + 7] >> 6;
       uint32_t prevL = 0xFFFFFFFFu;
@@ -353,35 +343,49 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const uint32_t sd = hz ? sdh : sdm;
             pre_c = hz ? kNoC : pre_c;
             const bool arr = (ust & kNotArrived) == kNotArrived;
-            const uint32_t k = (ust >> kKShift) & 7u;
-            const uint32_t kind = (ust >> (kKindShift + 2 * k)) & 3u;
-            const uint32_t r = sd & 0xFFFFu, used = ust & kUsedMask;
-            const uint32_t nd = arr ? used : (sd >> 16);  // d_0 before arrival
-            const bool isA = !arr && kind == CONVGPU_OP_ALLOC;
-            const bool isF = !arr && kind == CONVGPU_OP_FREE;
-            const bool isX = !arr && kind == CONVGPU_OP_FINISH;
-            const bool tnone = target == kNoC, ctg = c == target;
-            const uint32_t a_c = (ust & kAdmitted) ? L : (ctg ? a_tg : 0u);
             // ARRIVE (Fig. 3b/3c; R2)
-            const uint32_t g = (arr && tnone) ? min(L, free_mem) : 0u;
+            const uint32_t g = (arr && target == kNoC) ? min(L, free_mem) : 0u;
             const bool vadm = arr && g == L;
             const bool vtgt = arr && !vadm && g > 0;
+            // An arrival whose first op has delta 0 (before arrival the used
+            // field holds d_0) is followed by that op at the same tick: the
+            // DISPATCH after an ARRIVE is empty (with a target free = 0 and the
+            // target's resume test is unchanged; without one nothing is paused)
+            // and (t, c) stays the least key, so both events are applied in
+            // this step, the op on the post-ARRIVE state.  The peaks need no
+            // intermediate sample: the ARRIVE changes no used memory, and
+            // cap - free only falls after it.
+            const bool fz = arr && (ust & kUsedMask) == 0u;
+            const bool op = !arr || fz;
+            events += fz ? 1u : 0u;
+            const uint32_t ust1 = arr ? ((vadm ? kAdmitted : 0u) | (ust & kKindsMask)) : ust;
+            const uint32_t tg1 = vtgt ? c : target;
+            const uint32_t k = (ust1 >> kKShift) & 7u;
+            const uint32_t kind = (ust1 >> (kKindShift + 2 * k)) & 3u;
+            const uint32_t r = sd & 0xFFFFu, used = ust1 & kUsedMask;
+            const uint32_t nd = (arr && !fz) ? (ust & kUsedMask) : (sd >> 16);  // d_0 / d_{k+1}
+            const bool isA = op && kind == CONVGPU_OP_ALLOC;
+            const bool isF = op && kind == CONVGPU_OP_FREE;
+            const bool isX = op && kind == CONVGPU_OP_FINISH;
+            const bool tnone = tg1 == kNoC, ctg = c == tg1;
+            const uint32_t a_c = (ust1 & kAdmitted) ? L : (vtgt ? g : (ctg ? a_tg : 0u));
             // ALLOC
-            const uint32_t need = used + r + ((ust & kFirst) ? 0u : ovh);
+            const uint32_t need = used + r + ((ust1 & kFirst) ? 0u : ovh);
             const bool rej = isA && need > L;                // R10
             const bool grant = isA && !rej && need <= a_c;
             const bool pause = isA && !rej && !grant;       // reply withheld
             // FREE (R11)
             const bool badfree = isF && r > used;
-            free_mem = free_mem - g + (isX ? a_c : 0u);
+            const uint32_t free1 = free_mem - g;
+            peak_res = max(peak_res, cap - free1);
+            free_mem = free1 + (isX ? a_c : 0u);
             used_total = used_total + (grant ? need - used : 0u) - ((isF && !badfree) ? r : 0u) -
                          (isX ? used : 0u);
-            peak_res = max(peak_res, cap - free_mem);
             peak_used = max(peak_used, used_total);
             if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
             const bool clear_tg = isX && ctg;               // R20
-            target = vtgt ? c : (clear_tg ? kNoC : target);
-            a_tg = vtgt ? g : (clear_tg ? 0u : a_tg);
+            target = clear_tg ? kNoC : tg1;
+            a_tg = clear_tg ? 0u : (vtgt ? g : a_tg);
             stg_if(adm_out + c, (t << 6) | rank, vadm);     // admission at arrival
             rank += vadm ? 1u : 0u;
             n_rej += rej ? 1u : 0u;
@@ -406,17 +410,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
 #endif
             }
             const bool adv = !isX && !pause && !badfree;
-            uint32_t nu = ust;
-            nu = grant ? ((ust & ~kUsedMask) | need | kFirst) : nu;
-            nu = (isF && !badfree) ? ust - r : nu;
-            nu = isX ? (ust & ~kUsedMask) : nu;
-            nu = pause ? (ust | kPaused) : nu;
-            nu = arr ? ((vadm ? kAdmitted : 0u) | (ust & kKindsMask)) : nu;
-            nu = (adv && !arr) ? nu + kKOne : nu;
+            uint32_t nu = ust1;
+            nu = grant ? ((ust1 & ~kUsedMask) | need | kFirst) : nu;
+            nu = (isF && !badfree) ? ust1 - r : nu;
+            nu = isX ? (ust1 & ~kUsedMask) : nu;
+            nu = pause ? (ust1 | kPaused) : nu;
+            nu = (adv && op) ? nu + kKOne : nu;
             AT(s_ust, c) = nu;
             kc = badfree ? kNoC : c;
             nkc = adv ? (((t + nd) << 6) | c) : (isX ? (kDone | t) : (kPausedKey | plink));
-            pfk = (adv && !arr) ? k + 1u : 0xFFu;
+            pfk = (adv && op) ? k + 1u : 0xFFu;
           }
         } else {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
