@@ -30,7 +30,11 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__warps_eligible.avg.per_cycle_active", "smsp__inst_executed.sum",
         "launch__registers_per_thread", "launch__occupancy_limit_shared_mem",
         "launch__occupancy_limit_registers", "launch__grid_size", "launch__block_size",
-        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sectors.sum"]
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sectors.sum",
+        "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active",
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed"]
 TO_BYTES = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 
 
@@ -77,6 +81,7 @@ def full(rep, tag, events_per_launch, traffic, workload, traces):
                            "warp_instructions_per_event": round(k.get("warp_instructions_per_event", 0), 2),
                            "issue_active_pct": float(k["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"]),
                            "active_lanes": float(k["smsp__thread_inst_executed_per_inst_executed.ratio"]["value"]),
+                           "alu_pipe_pct": float(k["sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active"]["value"]),
                            "top_stalls": k["stall_share_top"]} for k in kernels}},
                       f, indent=1)
 
