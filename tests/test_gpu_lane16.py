@@ -135,3 +135,65 @@ def test_lane16_rejects_unsupported_shapes(cg):
         cg.replay(tr, w2.cap, "fifo", cg.alloc_out(64, 64, full=False), kernel="lane16")
     with pytest.raises(cg.ConvgpuError):  # R1-LIT runs on the warp kernel only
         cg.replay(tr, w2.cap, "fifo+literal", cg.alloc_out(64, 64), kernel="lane16")
+
+
+def _fused_arrival_batch(seed, count, cap, ovh):
+    """Input recipe aimed at the compact kernel's fused arrival step (an
+    arrival and its first op applied together when d_0 = 0): many arrivals
+    at the same tick, d_0 = 0 for 90 % of containers, first ops of every kind
+    with sizes at the boundaries (0, 1, the limit, one over it), limits 0 and
+    cap included, and a small capacity so arrivals find a partial target, no
+    target with free = 0, or a full ledger."""
+    rng = np.random.default_rng(seed)
+    n, K = 64, 4
+    arrival = np.cumsum(rng.choice([0, 0, 0, 1, 2], size=(count, n)), axis=1).astype(np.uint32)
+    lim_menu = np.array([0, 1, cap // 8, cap // 4, cap // 2, cap - 1, cap], np.int64)
+    limit = np.where(rng.random((count, n)) < 0.7, lim_menu[rng.integers(0, len(lim_menu), (count, n))],
+                     rng.integers(0, cap + 1, (count, n))).astype(np.uint32)
+    delta = rng.integers(0, 6, (count, K, n)).astype(np.uint32)
+    delta[:, 0, :] = np.where(rng.random((count, n)) < 0.9, 0, rng.integers(1, 4, (count, n)))
+    arg = np.zeros((count, K, n), np.uint32)
+    for i in range(count):
+        bad = rng.random() < 0.1  # this trace may free more than it holds
+        for c in range(n):
+            L = int(limit[i, c])
+            used = 0
+            for k in range(K - 1):
+                r = rng.random()
+                if r < 0.6:
+                    room = max(L - ovh - used, 0)
+                    sz = int(rng.choice([0, 1, room, room + 1, room // 2, int(rng.integers(0, room + 1))]))
+                    kind = W.ALLOC
+                    used += sz if sz <= room else 0
+                elif r < 0.75:
+                    sz = int(rng.choice([0, 1, used, used + 1] if bad else [0, used // 2, used]))
+                    sz = sz if (bad or sz <= used) else used
+                    kind = W.FREE
+                    used -= min(sz, used)
+                else:
+                    sz, kind = 0, W.NOP
+                arg[i, k, c] = W.op(kind, sz)
+            arg[i, K - 1, c] = W.op(W.FINISH)
+    return W.Batch(n, K, arrival, limit, delta, arg)
+
+
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("cap,ovh", [(64, 0), (200, 3), (1000, 0)])
+def test_lane16_fused_arrival_step(cg, orc, policy, cap, ovh):
+    """Element-by-element parity on traces built to hit every branch of the
+    fused arrival step: grant / reject / pause (as the new partial target, as
+    a zero-assignment newcomer behind a target, and with no target and free =
+    0, which triggers a selection), FREE at arrival (0 = valid, 1 = the
+    INVALID_FREE stop), NOP, zero limits (admitted on arrival with nothing
+    assigned) and same-tick arrival runs."""
+    b = _fused_arrival_batch(900 + cap + ovh, 600, cap, ovh)
+    base = 123_456_789 + cap
+    ref = orc.replay_batch(b, cap, policy, tid_base=base, rand_seed=17 + cap, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=base)
+    out = _gpu_replay(cg, tr, cap, policy, seed=17 + cap, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    # the batch must exercise the cases it is meant for
+    flags = ref["flags"]
+    assert (flags & 8).any() and (flags == 0).sum() > 100
+    assert int(ref["stats"]["n_select"]) > 0 and int(ref["stats"]["n_rejected"]) > 0
