@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--outputs", default="full", choices=["full", "summary"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane", "lane16"])
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-chunk", type=int, default=1 << 15, help="traces per host-path chunk")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=32768, help="traces per policy (cpu leg)")
@@ -280,7 +281,7 @@ def run_ours(args, rank, local_rank, world):
     def kernel_of(p):  # the rule of abi.cu launch_any / auto_variant
         if args.kernel != "auto":
             return args.kernel
-        if Nr < sms * 2 * 64 * 4:
+        if Nr < sms * 128:
             return "warp"
         return "lane16" if (full and n == 64 and K == 4) else "lane"
     launches_per_replay = {p: 2 if kernel_of(p) == "lane16" else 1 for p in POLICIES}
@@ -347,7 +348,7 @@ def run_ours(args, rank, local_rank, world):
 
     # e2e: the same metric through the host-memory C-ABI entry point
     if not args.no_e2e and not args.profile:
-        chunk = 1 << 17
+        chunk = args.e2e_chunk
         hbuf = [torch.empty(t.shape, dtype=torch.int32, pin_memory=True)
                 for t in (tr.arrival, tr.limit, tr.op_delta, tr.op_arg)]
         for h, t in zip(hbuf, (tr.arrival, tr.limit, tr.op_delta, tr.op_arg)):

@@ -283,7 +283,7 @@ def replay(traces: Traces, capacity: int, policy, out: ReplayOut, rand_seed: int
 
 
 def replay_host(arrival, limit, delta, arg, capacity: int, policies=("fifo",), *,
-                trace_id_base=0, rand_seed=0, ovh=0, chunk: int = 1 << 17,
+                trace_id_base=0, rand_seed=0, ovh=0, chunk: int = 1 << 15,
                 summary: Optional[np.ndarray] = None, workspace=None, stream=None,
                 kernel: str = "auto"):
     """End-to-end replay from HOST arrays (numpy or pinned torch; uint32/int32

@@ -84,15 +84,18 @@ bool use_bulk(const convgpu::ReplayArgs& a) {
          aligned16(a.arg);
 }
 
-// Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, profiles/):
-// lane-per-trace keeps 32 traces per warp in flight and needs enough traces
-// to give every SM several CTAs; below that warp-per-trace keeps more SMs
-// busy.  (policy is accepted for per-policy tuning; all four currently agree.)
+// Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, config [2]):
+// lane-per-trace holds 18,944 (32-bit) / 37,888 (compact) traces in flight
+// and replays one "round" of them in ~0.16 / ~0.27 ms; warp-per-trace holds
+// 4,736 and needs ~28 us per 1,000 traces.  From 128 traces per SM up, a
+// single partial lane round already beats the warp kernel (>= 2x at that
+// size); below it warp-per-trace keeps more SMs busy.  (policy is accepted
+// for per-policy tuning; all four currently agree.)
 uint32_t auto_variant(uint64_t count, int policy) {
   (void)policy;
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const bool big = count >= (uint64_t)sms * 2 * convgpu::kLptThreads * 4;
+  const bool big = count >= (uint64_t)sms * 128u;
   return big ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
 }
 
@@ -246,16 +249,22 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
   // kernel keeps them here during a replay (launches are stream-ordered)
   uint32_t* adm_scratch = (uint32_t*)(w + (size_t)np * stb);
 
-  cudaStream_t copy = nullptr;
+  // inputs go in on `copy`, summaries come back on `back` (PCIe is full
+  // duplex: the read-back of chunk j overlaps the copy-in of chunk j + 2)
+  cudaStream_t copy = nullptr, back = nullptr;
   cudaEvent_t h2d[2] = {nullptr, nullptr}, kdone[2] = {nullptr, nullptr};
-  cudaEvent_t start_ev = nullptr, copy_done = nullptr;
+  cudaEvent_t d2h[2] = {nullptr, nullptr};
+  cudaEvent_t start_ev = nullptr, copy_done = nullptr, back_done = nullptr;
   cudaError_t e = cudaStreamCreateWithFlags(&copy, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&back, cudaStreamNonBlocking);
   for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
     e = cudaEventCreateWithFlags(&h2d[b], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&kdone[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&d2h[b], cudaEventDisableTiming);
   }
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&copy_done, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&back_done, cudaEventDisableTiming);
   const uint64_t nchunks = (n + chunk - 1) / chunk;
   auto enqueue_h2d = [&](uint64_t j) -> cudaError_t {
     const int b = (int)(j & 1);
@@ -279,6 +288,8 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
     if (j + 1 < nchunks) e = enqueue_h2d(j + 1);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, h2d[b], 0);
+    // summary buffers b: read back (chunk j - 2) before they are rewritten
+    if (e == cudaSuccess && host_summary && j >= 2) e = cudaStreamWaitEvent(cs, d2h[b], 0);
     if (e != cudaSuccess) break;
     convgpu_traces_t dt = *ht;
     dt.arrival = arr[b]; dt.limit = lim[b]; dt.op_delta = del[b]; dt.op_arg = arg[b];
@@ -292,10 +303,11 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     }
     if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
     if (e == cudaSuccess && host_summary) {
-      e = cudaStreamWaitEvent(copy, kdone[b], 0);
+      e = cudaStreamWaitEvent(back, kdone[b], 0);
       for (int q = 0; q < np && e == cudaSuccess; ++q)
         e = cudaMemcpyAsync(host_summary + (uint64_t)q * n + lo, sum[b][q],
-                            cnt * sizeof(convgpu_summary_t), cudaMemcpyDeviceToHost, copy);
+                            cnt * sizeof(convgpu_summary_t), cudaMemcpyDeviceToHost, back);
+      if (e == cudaSuccess) e = cudaEventRecord(d2h[b], back);
     }
   }
   for (int q = 0; q < np && e == cudaSuccess; ++q)
@@ -305,14 +317,19 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
   // then bracket every copy and kernel of the call)
   if (e == cudaSuccess) e = cudaEventRecord(copy_done, copy);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, copy_done, 0);
+  if (e == cudaSuccess) e = cudaEventRecord(back_done, back);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, back_done, 0);
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
   for (int b = 0; b < 2; ++b) {
     if (h2d[b]) cudaEventDestroy(h2d[b]);
     if (kdone[b]) cudaEventDestroy(kdone[b]);
+    if (d2h[b]) cudaEventDestroy(d2h[b]);
   }
   if (start_ev) cudaEventDestroy(start_ev);
   if (copy_done) cudaEventDestroy(copy_done);
+  if (back_done) cudaEventDestroy(back_done);
   if (copy) cudaStreamDestroy(copy);
+  if (back) cudaStreamDestroy(back);
   return e == cudaSuccess ? 0 : fail_cuda(e, "replay_host");
 }
 
