@@ -1,11 +1,12 @@
-"""Small replay of every kernel variant / policy (incl. the literal reading)
-and the NEXT-3 wrapper kernel for compute-sanitizer runs: memcheck,
+"""Small replay of every kernel variant / policy (incl. the literal reading),
+the host-memory path and the NEXT-3 wrapper kernel for compute-sanitizer runs: memcheck,
 racecheck, synccheck, initcheck."""
 import os
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import paper_conf_cluster_kangjkkk17_b200 as cg  # noqa: E402
@@ -28,6 +29,26 @@ tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
 for kernel in ("warp", "lane"):
     for pol in W.POLICIES:
         cg.replay(tr, 16, pol, cg.alloc_out(200, 7), ovh=2, kernel=kernel)
+torch.cuda.synchronize()
+# the compact lane-per-trace kernel (n = 64, K = 4): config [2] (+ rho 8, whose
+# limits exceed 16 bits and go through the marked 32-bit fallback launch) and
+# a mixed edge-case batch with context overhead
+for w in (W.CONFIGS["c2"], W.rho_sweep(8, rand_seed=3)):
+    tr = cg.generate(w.gen, 0, 700)
+    for pol in W.POLICIES:
+        cg.replay(tr, w.cap, pol, cg.alloc_out(700, 64, range_count=1, range_size=1 << 20),
+                  rand_seed=3, ovh=w.ovh, kernel="lane16")
+b = W.random_batch(6, 300, 64, 4, 64, ovh=1, mode="mixed", limit_choices=range(0, 65))
+tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
+for pol in W.POLICIES:
+    cg.replay(tr, 64, pol, cg.alloc_out(300, 64), ovh=1, kernel="lane16")
+torch.cuda.synchronize()
+# the host-memory path (two copy streams, double-buffered chunks, AUTO kernel)
+w = W.CONFIGS["c2"]
+g = cg.generate(w.gen, 0, 40_000)
+h = [t.cpu() for t in (g.arrival, g.limit, g.op_delta, g.op_arg)]
+summ = np.zeros((4, 40_000), cg.SUMMARY_DTYPE)
+cg.replay_host(*h, w.cap, W.POLICIES, chunk=19_000, summary=summ, rand_seed=3)
 torch.cuda.synchronize()
 # NEXT-3 wrapper kernel: the n = 64 / K = 4 fast path, K = 4 and generic shapes
 import numpy as np  # noqa: E402
