@@ -57,6 +57,24 @@ __device__ __forceinline__ uint32_t ffs64(uint32_t lo, uint32_t hi) {  // lowest
 __device__ __forceinline__ uint32_t fls64(uint32_t lo, uint32_t hi) {  // highest set bit
   return hi ? 63u - (uint32_t)__clz(hi) : 31u - (uint32_t)__clz(lo);
 }
+// position of the j-th (0-based) set bit of (hi:lo), j < popc: a branch-free
+// popc binary search (the __fns intrinsic is a branchy software sequence,
+// and two of them behind a lo/hi branch diverge inside a warp)
+__device__ __forceinline__ uint32_t nth_set64(uint32_t lo, uint32_t hi, uint32_t j) {
+  const uint32_t cl = (uint32_t)__popc(lo);
+  const bool up = j >= cl;
+  uint32_t w = up ? hi : lo, pos = up ? 32u : 0u;
+  j -= up ? cl : 0u;
+#pragma unroll
+  for (uint32_t s = 16; s >= 1; s >>= 1) {
+    const uint32_t c = (uint32_t)__popc(w & ((1u << s) - 1u));
+    const bool b = j >= c;
+    j -= b ? c : 0u;
+    pos += b ? s : 0u;
+    w = b ? (w >> s) : w;
+  }
+  return pos;
+}
 __device__ __forceinline__ void lowmask64(uint32_t r, uint32_t& lo, uint32_t& hi) {  // bits < r
   lo = r >= 32 ? 0xFFFFFFFFu : ((1u << r) - 1u);
   hi = r >= 64 ? 0xFFFFFFFFu : (r <= 32 ? 0u : ((1u << (r - 32)) - 1u));

@@ -559,7 +559,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
                                          (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
               ++draws;
               const uint32_t jj = __umulhi(x.x, m);
-              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+              sel = lpt::nth_set64(pm_lo, pm_hi, jj);
             }
             target = sel;
             a_tg = 0;

@@ -467,7 +467,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
                                          (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
               ++draws;
               const uint32_t jj = __umulhi(x.x, m);
-              sel = (jj < clo) ? __fns(pm_lo, 0, jj + 1) : 32u + __fns(pm_hi, 0, jj - clo + 1);
+              sel = lpt::nth_set64(pm_lo, pm_hi, jj);
             }
             target = sel;
             a_tg = 0;
