@@ -100,8 +100,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   uint32_t* const s_key = W0 + lane;
   uint32_t* const s_ust = W0 + 1 * n * 32 + lane;
   uint32_t* const s_sd = W0 + 2 * n * 32 + lane;
-  uint32_t* const s_Lw = W0 + 3 * n * 32 + lane;
-  uint16_t* const s_L = reinterpret_cast<uint16_t*>(s_Lw);
+  // limits: u16 of container c of this lane at [c * 32 + lane] (one IMAD per
+  // address; at most 2-way bank conflicts, between lanes 2j and 2j + 1)
+  uint16_t* const s_L = reinterpret_cast<uint16_t*>(W0 + 3 * n * 32) + lane;
   // Best-Fit: rank of container c in (L, index) order and container of rank
   // r, bytes (byte e of this lane at [(e >> 2) * 128 + (e & 3)])
   uint8_t* const s_rof = reinterpret_cast<uint8_t*>(W0 + (3 * n + n / 2) * 32) + lane * 4;
@@ -109,7 +110,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // staging slot of the one-op-ahead fetch: {op word, delta of the op after}
   uint32_t* const s_stg = W0 + (3 * n + n / 2 + extra_bytes(POLICY) / 4) * 32 + lane;
 #define AT(arr, c) (arr)[(c) * 32u]
-#define LIM(c) s_L[((c) >> 1) * 64u + ((c) & 1u)]
+#define LIM(c) s_L[(c) * 32u]
 #define ROF(c) s_rof[((c) >> 2) * 128u + ((c) & 3u)]
 #define PI(r) s_pi[((r) >> 2) * 128u + ((r) & 3u)]
 
@@ -171,7 +172,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       uint4 d4[4], w4[4];
 #pragma unroll
       for (int k = 0; k < 4; ++k) { d4[k] = __ldg(D4 + k * 16 + q); w4[k] = __ldg(R4 + k * 16 + q); }
-      uint32_t lp[2] = {0, 0};
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const uint32_t c = 4 * q + j, a = comp(a4, j), L = comp(l4, j);
@@ -194,13 +194,12 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         AT(s_key, c) = key;
         AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu);
         AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
-        lp[j >> 1] |= min(L, 0xFFFFu) << (16 * (j & 1));
+        LIM(c) = (uint16_t)min(L, 0xFFFFu);
         gmin[c >> 3] = min(gmin[c >> 3], key);
         base[c] = bsum;
         if (c == 0) arr0 = a;
       }
-      s_Lw[(2 * q) * 32] = lp[0];
-      s_Lw[(2 * q + 1) * 32] = lp[1];
+
     }
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     // not representable in the 16-bit fields: the 32-bit kernel replays it
