@@ -1,0 +1,66 @@
+"""bench.py's driver contract, on CPU: the reference arm (the C oracle timed
+on the host cores) prints one JSON line with BASELINE.json's metric and the
+keys the contract names, alone and under a 2-rank torchrun (rank 0 prints,
+the other rank exits 0 without work); our arm has no CPU fallback, so on a
+host without a GPU it exits non-zero and prints no result line."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+BENCH = os.path.join(ROOT, "bench.py")
+
+
+def _metric():
+    with open(os.path.join(ROOT, "BASELINE.json")) as f:
+        return json.load(f)["metric"]
+
+
+def _json_lines(out):
+    return [json.loads(l) for l in out.splitlines() if l.startswith("{")]
+
+
+def _check_reference_line(d, n_gpus):
+    assert d["impl"] == "reference" and d["metric"] == _metric()
+    assert d["unit"] == "events/s" and d["higher_is_better"] is True and d["value"] > 0
+    assert d["n_gpus"] == n_gpus and d["steps"] == 1 and d["warmup"] == 1
+    cb = d["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] == 1 and cb["value"] == d["value"] and cb["sample"]
+    e = d["e2e"]
+    assert e["value"] == d["value"] and e["unit"] == d["unit"]
+    assert e["h2d_bytes_per_step"] == 0 and e["d2h_bytes_per_step"] == 0
+    assert d["config"]["workload"] == "c2_1e6x64_rho2"
+
+
+def test_reference_arm_json_line():
+    r = subprocess.run([sys.executable, BENCH, "--impl", "reference", "--steps", "1", "--warmup", "1",
+                        "--ref-sample", "64"], capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1
+    _check_reference_line(lines[0], 1)
+
+
+def test_reference_arm_two_ranks():
+    env = dict(os.environ, OMP_NUM_THREADS="1")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29517", BENCH, "--impl", "reference",
+                        "--gpus", "2", "--steps", "1", "--warmup", "1", "--ref-sample", "64"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1  # rank 0 only
+    _check_reference_line(lines[0], 2)
+
+
+def test_our_arm_has_no_cpu_fallback():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is visible: the CUDA path would run")
+    r = subprocess.run([sys.executable, BENCH, "--steps", "1", "--warmup", "3", "--no-e2e",
+                        "--no-cpu-baseline"], capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode != 0
+    assert not _json_lines(r.stdout)
