@@ -126,31 +126,55 @@ class ClockSampler:
                 "samples": len(self.rows), "samples_under_load": len(loaded)}
 
 
-# ------------------------------------------------------------------ reference arm
-def run_reference(args, rank, world):
-    """The oracle (plain single-threaded C) timed on this host's cores."""
-    if rank != 0:
-        return
+# ------------------------------------------------------------------ oracle timing
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def oracle_run(w, traces: int, threads: int) -> tuple:
+    """Replay global ids [0, traces) under every policy with the C oracle as it
+    stands (single-threaded code), on `threads` host threads over disjoint id
+    ranges (the ctypes call releases the GIL; every replay keeps its state on
+    its own stack).  Returns (events, seconds)."""
     import oracle
-    w = W.CONFIGS[args.workload]
-    S = args.ref_sample
+    from concurrent.futures import ThreadPoolExecutor
     oracle.build()
     oracle.lib()
+    cuts = [traces * j // threads for j in range(threads + 1)]
+    jobs = [(p, cuts[j], cuts[j + 1]) for p in POLICIES for j in range(threads) if cuts[j + 1] > cuts[j]]
+    run = lambda j: oracle.replay_range(w, j[0], j[1], j[2])["stats"]["events"]  # noqa: E731
+    t0 = time.perf_counter()
+    if threads == 1:
+        ev = sum(run(j) for j in jobs)
+    else:
+        with ThreadPoolExecutor(threads) as ex:
+            ev = sum(ex.map(run, jobs))
+    return ev, time.perf_counter() - t0
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    """The oracle (plain single-threaded C) timed on this host's cores: one
+    oracle thread per core, each on its own slice of the step's traces."""
+    if rank != 0:
+        return
+    w = W.CONFIGS[args.workload]
+    C = host_cores()
+    S = args.ref_sample * C
     times = []
     events = 0
     for step in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        ev = 0
-        for p in POLICIES:
-            r = oracle.replay_range(w, p, 0, S)
-            ev += r["stats"]["events"]
-        dt = time.perf_counter() - t0
+        ev, dt = oracle_run(w, S, C)
         if step >= args.warmup:
             times.append(dt)
             events += ev
     total = sum(times)
     value = events / total
-    sample = f"{S} traces x {len(POLICIES)} policies per step of {w.name} (ids 0..{S - 1})"
+    sample = (f"{S} traces x {len(POLICIES)} policies per step of {w.name} (ids 0..{S - 1}), "
+              f"{C} oracle threads on disjoint id ranges")
     out = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "events/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
@@ -159,7 +183,7 @@ def run_reference(args, rank, world):
         "config": {"workload": w.name, "traces_per_step": S, "containers": w.gen.n,
                    "ops_per_container": w.gen.K, "capacity_mib": w.cap,
                    "policies": list(POLICIES)},
-        "cpu_baseline": {"value": value, "unit": "events/s", "cores": 1, "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": "events/s", "cores": C, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
@@ -169,16 +193,17 @@ def run_reference(args, rank, world):
 
 # ------------------------------------------------------------------ our arm
 def cpu_baseline(w, sample):
-    import oracle
-    oracle.build()
-    t0 = time.perf_counter()
-    ev = 0
-    for p in POLICIES:
-        ev += oracle.replay_range(w, p, 0, sample)["stats"]["events"]
-    dt = time.perf_counter() - t0
-    return {"value": ev / dt, "unit": "events/s", "cores": 1, "kind": "oracle",
-            "sample": f"{sample} traces x {len(POLICIES)} policies of {w.name} "
-                      f"(ids 0..{sample - 1}), single-threaded C oracle, {dt:.1f} s"}
+    """The oracle on all host cores (a bounded sample: `sample` traces per core
+    and policy), and on one core (`sample` traces per policy)."""
+    C = host_cores()
+    ev1, dt1 = oracle_run(w, sample, 1)
+    evc, dtc = oracle_run(w, sample * C // 2, C)
+    return {"value": evc / dtc, "unit": "events/s", "cores": C, "kind": "oracle",
+            "sample": f"{sample * C // 2} traces x {len(POLICIES)} policies of {w.name} "
+                      f"(ids 0..{sample * C // 2 - 1}), {C} threads of the single-threaded C "
+                      f"oracle on disjoint id ranges, {dtc:.1f} s",
+            "single_core": {"value": ev1 / dt1, "cores": 1,
+                            "sample": f"{sample} traces x {len(POLICIES)} policies, {dt1:.1f} s"}}
 
 
 def ncu_summary(workload, traces):
