@@ -7,7 +7,7 @@
 //  * 14 bytes per container instead of 24 (n = 64: 896 B per trace, 28 KB per
 //    warp): key (u32), ust (u32: used 16 | op index 3 | FIRST | PAUSED |
 //    ADMITTED | op kinds 2 x K), sd (u32: size of the current op, saturated
-//    to 16 bits | delta of the next op 16), L (u16);
+//    to 16 bits | delta of the next op 16), L (u16, [container][lane]);
 //  * no admission word: an admission is stored straight to admit_tick (as
 //    tick << 6 | rank) and read back by the epilogue; the finish tick lives
 //    in the container's key after FINISH (0x80000000 | tick) and a paused
@@ -16,6 +16,8 @@
 //    memory), both above every event key (ticks < 2^25 here);
 //  * Best-Fit keeps two bytes per container (rank of (L, index), container of
 //    rank) and the "same limit as the previous rank" bits in two registers;
+//  * an arrival whose first op has delta 0 is applied together with that op
+//    in one step (see the EVENT step);
 //  * the one-op-ahead fetch (raw op word + next delta, cp.async) lands in a
 //    2-word staging slot and is packed into the container's sd word at the
 //    end of the NEXT iteration, so the copy has a whole iteration to land
