@@ -576,14 +576,23 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
 
 template <int POLICY>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
-  const int threads = 32 * warps_per_cta(POLICY);
-  const size_t smem = (size_t)threads * lane_bytes(POLICY);
   auto kern = replay_lpt16_kernel<POLICY>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
   int dev = 0, sms = 0;
+  cudaError_t e;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  // one persistent CTA per SM; a batch smaller than one trace per lane of a
+  // full grid gets smaller CTAs, so that it still spreads over every SM
+  uint64_t warps = (uint64_t)warps_per_cta(POLICY);
+  if (!a.grid_override) {
+    const uint64_t w = (a.count + 32ull * sms - 1) / (32ull * sms);
+    warps = w < 1 ? 1 : (w < warps ? w : warps);
+  }
+  const int threads = (int)(32 * warps);
+  const size_t smem = (size_t)threads * lane_bytes(POLICY);
+  if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)((size_t)32 * warps_per_cta(POLICY) * lane_bytes(POLICY)))) != cudaSuccess)
+    return e;
   const uint64_t need = (a.count + threads - 1) / threads;
   uint64_t grid = (uint64_t)sms;  // one CTA per SM, persistent
   if (a.grid_override) grid = a.grid_override;
