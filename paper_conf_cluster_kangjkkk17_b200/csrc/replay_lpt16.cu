@@ -519,7 +519,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           sts_if(&AT(s_key, kcs), nkc, kc != kNoC);
           regroup(kcs);
           // retire last iteration's fetch (issued one iteration ago)
-          lpt::cp_wait0_if(pre_c != kNoC);
+          lpt::cp_wait0();  // nothing pending if nothing was fetched: no branch needed
           sts_if(&AT(s_sd, pre_c & 63u), pack_sd(AT(s_stg, 0), AT(s_stg, 1)), pre_c != kNoC);
           // op k word and the delta of op k+1 (clamped: FINISH never reads it)
           const bool f = pfk < K;
