@@ -306,7 +306,7 @@ def run_ours(args, rank, local_rank, world):
     def kernel_of(p):  # the rule of abi.cu launch_any / auto_variant
         if args.kernel != "auto":
             return args.kernel
-        if Nr < sms * 128:
+        if Nr < sms * 40:
             return "warp"
         return "lane16" if (full and n == 64 and K == 4) else "lane"
     launches_per_replay = {p: 2 if kernel_of(p) == "lane16" else 1 for p in POLICIES}

@@ -84,18 +84,18 @@ bool use_bulk(const convgpu::ReplayArgs& a) {
          aligned16(a.arg);
 }
 
-// Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, config [2]):
-// lane-per-trace holds 18,944 (32-bit) / 37,888 (compact) traces in flight
-// and replays one "round" of them in ~0.16 / ~0.27 ms; warp-per-trace holds
-// 4,736 and needs ~28 us per 1,000 traces.  From 128 traces per SM up, a
-// single partial lane round already beats the warp kernel (>= 2x at that
-// size); below it warp-per-trace keeps more SMs busy.  (policy is accepted
-// for per-policy tuning; all four currently agree.)
+// Kernel choice for CONVGPU_KERNEL_AUTO (measured on B200, config [2] traces,
+// scripts/gpu_small.sh): a lane-per-trace launch costs one "round" (~0.17-
+// 0.24 ms per policy) for any batch up to its 18,944 (32-bit) / 37,888
+// (compact) lanes; warp-per-trace holds 4,736 traces in flight at ~0.16 ms
+// per 4,736.  Crossover ~40 traces per SM: warp-per-trace at 1,000-4,736
+// traces (0.09-0.16 vs 0.17-0.24 ms), lane kernels 2x faster from 9,472.
+// (policy is accepted for per-policy tuning; all four currently agree.)
 uint32_t auto_variant(uint64_t count, int policy) {
   (void)policy;
   int dev = 0, sms = 148;
   if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const bool big = count >= (uint64_t)sms * 128u;
+  const bool big = count >= (uint64_t)sms * 40u;
   return big ? CONVGPU_KERNEL_LANE_PER_TRACE : CONVGPU_KERNEL_WARP_PER_TRACE;
 }
 
