@@ -355,3 +355,23 @@ def test_extreme_values(cg, orc, kernel, policy, nk):
     out = _gpu_replay(cg, tr, cap, policy, seed=2**64 - 1, ovh=ovh, kernel=kernel)
     _compare(cg, out, ref)
     _compare_stats(cg, out, ref["stats"])
+
+
+def test_replay_host_production_chunks(cg, orc):
+    """The host path as bench.py's e2e leg runs it: default 32,768-trace chunks
+    (compact lane kernel, two copy streams), a short tail chunk (warp kernel
+    below 40 traces per SM), every policy on each resident chunk.  Every
+    trace's summary is compared with the oracle's, field by field."""
+    w = W.CONFIGS["c2"]
+    base, N = 3_000_000, 2 * 32768 + 3001
+    A, L, D, R = orc.generate_batch(w.gen, base, N)
+    summ = np.zeros((4, N), cg.SUMMARY_DTYPE)
+    st = cg.replay_host(A, L, D, R, w.cap, POLS, trace_id_base=base, summary=summ,
+                        rand_seed=w.rand_seed)
+    for q, pol in enumerate(POLS):
+        ref = orc.replay_range(w, pol, base, base + N)
+        for f in SUMMARY_FIELDS:
+            np.testing.assert_array_equal(summ[q][f], ref[f].astype(summ[q][f].dtype),
+                                          err_msg=f"{pol} {f}")
+        for k, v in ref["stats"].items():
+            assert cg.stats_dict(st[q])[k] == v, (pol, k)
