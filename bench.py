@@ -206,6 +206,14 @@ def cpu_baseline(w, sample):
                             "sample": f"{sample} traces x {len(POLICIES)} policies, {dt1:.1f} s"}}
 
 
+def measured_sm_mhz() -> float:
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["sm_max_mhz"])
+    except Exception:
+        return 1965.0  # B200 max SM clock (B200_PROFILING.md)
+
+
 def ncu_summary(workload, traces):
     """DRAM bytes per replay launch and the limiter evidence from the committed
     ncu --set full summary (profiles/ncu_full_summary.json), if it matches."""
@@ -346,6 +354,29 @@ def run_ours(args, rank, local_rank, world):
                         "rate is limited by each trace's serial event chain (latency / issue), "
                         "see ncu_limiter and DESIGN.md §6.4"}
 
+    # secondary roofline: instruction issue (the binding limit, DESIGN.md
+    # §6.4): live events/s x the warp instructions per event of the same
+    # kernel in the committed ncu capture, against 4 issue slots per SM per
+    # clock (B200: 148 SMs at the measured max SM clock)
+    issue = None
+    lim = ncu.get("limiter") or {}
+    ipe = {}
+    for p in POLICIES:
+        pid = {"fifo": 0, "best_fit": 1, "recent_fit": 2, "random_fit": 3}[p]
+        for kname, v in lim.items():
+            if kernel_of(p) == "lane16" and f"replay_lpt16_kernel<{pid}>" in kname:
+                ipe[p] = v
+    if len(ipe) == len(POLICIES):
+        inst = sum(ipe[p]["warp_instructions_per_event"] * Nr * per_trace_events for p in POLICIES)
+        t_s = sum(launch_ms.values()) / 1e3
+        sm_mhz = (clocks or {}).get("sm_mhz") or measured_sm_mhz()  # median under load
+        peak_issue = sms * 4 * sm_mhz * 1e6
+        issue = {"bound": "alu", "achieved": inst / t_s, "peak": peak_issue, "unit": "warp-inst/s",
+                 "frac": inst / t_s / peak_issue,
+                 "alu_pipe_pct": {p: ipe[p].get("alu_pipe_pct") for p in POLICIES},
+                 "source": "ncu warp instructions per event (" + str(ncu.get("source")) + ") x live "
+                           "launch times; peak = SMs x 4 schedulers x 1 instr/clk x SM clock under load"}
+
     result = None
     if rank == 0:
         result = {
@@ -367,6 +398,7 @@ def run_ours(args, rank, local_rank, world):
             "gen_ms": gen_ms,
             "gen_write_gbs": Nr * in_b / (gen_ms / 1e3) / 1e9,
             "roofline": roofline,
+            "issue_roofline": issue,
             "gpu_launches": args.steps * sum(launches_per_replay.values()),
             "clocks": clocks,
         }
