@@ -321,11 +321,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     do {
       if (have && !tdone) {
         uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
-        if (!dmode) {
+        // next event (a2).  If it belongs to the container whose next op was
+        // fetched in the previous iteration (rare), this lane idles for one
+        // iteration: the tail below retires that fetch into the container's
+        // sd word, so the event block never handles an op still in flight.
+        const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
+        const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
+        const uint32_t kmin = min(min(m01, m23), min(m45, m67));
+        const bool hz = (kmin & 63u) == pre_c && kmin < kDone;
+        if (!dmode && !hz) {
           // ================= EVENT step (a2 + a3), branch-free =================
-          const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
-          const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
-          const uint32_t kmin = min(min(m01, m23), min(m45, m67));
           if (kmin >= kDone) {
             if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
             tdone = true;
@@ -333,16 +338,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const uint32_t t = kmin >> 6, c = kmin & 63u;
             cur_t = t;
             ++events;
-            // the container fetched in the previous iteration: its op data are
-            // still in registers (rare: warp-uniform slow path)
-            // (predicated: wait, take the staged copy, store it, drop the retire)
-            const bool hz = c == pre_c;
-            lpt::cp_wait0_if(hz);
-            const uint32_t sdh = pack_sd(AT(s_stg, 0), AT(s_stg, 1));
-            sts_if(&AT(s_sd, c), sdh, hz);
-            const uint32_t ust = AT(s_ust, c), sdm = AT(s_sd, c), L = LIM(c);
-            const uint32_t sd = hz ? sdh : sdm;
-            pre_c = hz ? kNoC : pre_c;
+            const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
             const bool arr = (ust & kNotArrived) == kNotArrived;
             // ARRIVE (Fig. 3b/3c; R2)
             const uint32_t g = (arr && target == kNoC) ? min(L, free_mem) : 0u;
@@ -422,7 +418,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             nkc = adv ? (((t + nd) << 6) | c) : (isX ? (kDone | t) : (kPausedKey | plink));
             pfk = (adv && op) ? k + 1u : 0xFFu;
           }
-        } else {
+        } else if (dmode) {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
           const uint32_t t = cur_t;
           if (POLICY == CONVGPU_FIFO) {
