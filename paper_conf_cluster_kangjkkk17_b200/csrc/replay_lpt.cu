@@ -395,11 +395,16 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
         uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
         const uint32_t pf = pfc;  // previous iteration's group
         pfc = kNoC;
-        if (!dmode) {
+        // next event (a2).  If it belongs to the container whose op words were
+        // fetched in the previous iteration (rare), this lane idles for one
+        // iteration; the cp.async.wait_group 1 of its next event step then
+        // covers that fetch (as in replay_lpt16.cu).
+        const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
+        const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
+        const uint32_t kmin = min(min(m01, m23), min(m45, m67));
+        const bool hz = (kmin & 63u) == pf && kmin != kKeyNone;
+        if (!dmode && !hz) {
           // ================= EVENT step (a2 + a3), branch-free =================
-          const uint32_t m01 = min(gmin[0], gmin[1]), m23 = min(gmin[2], gmin[3]);
-          const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
-          const uint32_t kmin = min(min(m01, m23), min(m45, m67));
           if (kmin == kKeyNone) {
             if (live) flags |= CONVGPU_FLAG_DEADLOCK;  // P:7
             tdone = true;
@@ -407,7 +412,6 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             const uint32_t t = kmin >> 6, c = kmin & 63u;
             cur_t = t;
             cp_wait1();  // every group but the previous iteration's is complete
-            cp_wait0_if(c == pf);
             ++events;
             const uint32_t ust = AT(s_ust, c), L = AT(s_L, c), cw = AT(s_cw, c);
             const uint32_t nd = AT(s_nd, c), am = AT(s_adm, c);
@@ -481,7 +485,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
             nkc = adv ? (((t + nd) << 6) | c) : kKeyNone;
             pfk = (adv && !arr) ? ((nu >> kKShift) & 7u) : 0xFFu;
           }
-        } else {
+        } else if (dmode) {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
           // A step = [SELECT if there is no fill target] + fill / resume / admit
           // of the target; an admit keeps the lane in dispatch mode (the
