@@ -116,8 +116,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
 #define ROF(c) s_rof[((c) >> 2) * 128u + ((c) & 3u)]
 #define PI(r) s_pi[((r) >> 2) * 128u + ((r) & 3u)]
 
+  // A warp replays 32 consecutive traces per round; round-robin warp slots
+  // run SM-first (slot = wib * gridDim + block), so the last, partial round
+  // spreads over every SM instead of filling the first CTAs.
   const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
-  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t i = ((uint64_t)wib * gridDim.x + blockIdx.x) * 32u + lane;
 
   unsigned long long st_traces = 0, st_events = 0, st_mk = 0, st_wait = 0, st_rej = 0,
                      st_sel = 0, st_dig = 0;
