@@ -108,6 +108,18 @@ __device__ __forceinline__ uint32_t redux_max(uint32_t v) {
 }
 
 // ---------------------------------------------------------------- kernel
+// A write to the per-warp scheduler state (the warp runs one trace with
+// warp-uniform control flow, so every lane holds the same value): the warp
+// syncs so every lane's earlier read of the location is done, one lane
+// stores, and the warp syncs again so every later read sees the store.
+#define WSTORE(lhs, val)                  \
+  do {                                    \
+    const auto wstore_v_ = (val);         \
+    __syncwarp();                         \
+    if (lane == 0) (lhs) = wstore_v_;     \
+    __syncwarp();                         \
+  } while (0)
+
 // NF: compile-time container count (64) or 0 = runtime p.n.
 // LIT: the literal re-select-on-every-release reading R1-LIT (NEXT-1).
 template <int POLICY, bool BULK, int NF, bool LIT>
@@ -250,15 +262,15 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
           if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
           uint32_t adm = kKeyNone;
           ust = 0;
-          if (LIT) ca[c] = g;
+          if (LIT) WSTORE(ca[c], g);
           if (g == L) {
             adm = (t << 6) | rank; ++rank; ust = kAdmitted;
           } else if (g > 0 && !LIT) {
             target = c; a_tg = g;
           }
           const uint32_t d1 = cx[c].x;
-          cx[c] = make_uint2(0u, adm);
-          cs[c] = make_uint4(ust, s.y, d1, L);
+          WSTORE(cx[c], make_uint2(0u, adm));
+          WSTORE(cs[c], make_uint4(ust, s.y, d1, L));
           nk = ((t + s.z) << 6) | c;
         } else {
           const uint32_t cw = s.y;
@@ -277,12 +289,12 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             } else {  // pause: reply withheld
               ust |= kPaused;
               const uint32_t wv = cx[c].x - t;
-              cx[c] = make_uint2(wv, POLICY == CONVGPU_RECENT_FIT ? seq : kKeyNone);
+              WSTORE(cx[c], make_uint2(wv, POLICY == CONVGPU_RECENT_FIT ? seq : kKeyNone));
               ++seq;
               if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
               adv = false;
               disp = LIT || (target == kTargetNone);
-              cs[c].x = ust;
+              WSTORE(cs[c].x, ust);
             }
           } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
             if (r > used) { flags |= CONVGPU_FLAG_INVALID_FREE; break; }
@@ -294,7 +306,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             used_total -= used;
             --live;
             if (c == target) { target = kTargetNone; a_tg = 0; }  // R20
-            cs[c] = make_uint4(ust & ~kUsedMask, cw, t, L);  // nd := finish tick
+            WSTORE(cs[c], make_uint4(ust & ~kUsedMask, cw, t, L));  // nd := finish tick
             adv = false;
             disp = true;
           }
@@ -304,7 +316,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             ust = (ust & ~kKMask) | (k << kKShift);
             const uint32_t ncw = R[k * n + c];
             const uint32_t nnd = (k + 1 < K) ? D[(k + 1) * n + c] : 0u;
-            cs[c] = make_uint4(ust, ncw, nnd, L);
+            WSTORE(cs[c], make_uint4(ust, ncw, nnd, L));
           }
         }
         key0 = (c == lane) ? nk : key0;
@@ -356,7 +368,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             const uint32_t Lx = st.w;
             const uint32_t g = min(free_mem, Lx - ca[x]);
             const uint32_t ax = ca[x] + g;
-            ca[x] = ax;
+            WSTORE(ca[x], ax);
             free_mem -= g;
             peak_res = max(peak_res, cap - free_mem);
             uint32_t ut = st.x;
@@ -366,7 +378,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
               if (uu + pend <= ax) {  // RESUME (R9)
                 used_total += pend;
                 peak_used = max(peak_used, used_total);
-                cx[x] = make_uint2(cx[x].x + t, kKeyNone);
+                WSTORE(cx[x], make_uint2(cx[x].x + t, kKeyNone));
                 if (x < 32) pm_lo &= ~(1u << x); else pm_hi &= ~(1u << (x - 32));
                 const uint32_t k = ((ut >> kKShift) & 7u) + 1u;
                 ut = (ut & ~(kUsedMask | kKMask | kPaused)) | (uu + pend) | kFirst | (k << kKShift);
@@ -378,8 +390,8 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
               }
             }
             if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
-            if (ax == Lx) { cx[x].y = (t << 6) | rank; ++rank; ut |= kAdmitted; }
-            cs[x] = make_uint4(ut, st.y, st.z, Lx);
+            if (ax == Lx) { WSTORE(cx[x].y, (t << 6) | rank); ++rank; ut |= kAdmitted; }
+            WSTORE(cs[x], make_uint4(ut, st.y, st.z, Lx));
           }
         } else if (disp) {
           for (;;) {
@@ -400,7 +412,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
                   used_total += pend;
                   peak_used = max(peak_used, used_total);
                   if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
-                  cx[tg] = make_uint2(cx[tg].x + t, kKeyNone);
+                  WSTORE(cx[tg], make_uint2(cx[tg].x + t, kKeyNone));
                   if (tg < 32) pm_lo &= ~(1u << tg); else pm_hi &= ~(1u << (tg - 32));
                   const uint32_t k = ((ut >> kKShift) & 7u) + 1u;
                   ut = (ut & ~(kUsedMask | kKMask | kPaused)) | (uu + pend) | kFirst | (k << kKShift);
@@ -412,13 +424,13 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
                 }
               }
               if (a_tg == Lt) {  // fully guaranteed: admit, cascade leftover
-                cx[tg].y = (t << 6) | rank; ++rank;
-                cs[tg] = make_uint4(ut | kAdmitted, st.y, st.z, Lt);
+                WSTORE(cx[tg].y, (t << 6) | rank); ++rank;
+                WSTORE(cs[tg], make_uint4(ut | kAdmitted, st.y, st.z, Lt));
                 target = kTargetNone;
                 a_tg = 0;
                 continue;
               }
-              cs[tg] = make_uint4(ut, st.y, st.z, Lt);
+              WSTORE(cs[tg], make_uint4(ut, st.y, st.z, Lt));
               break;
             }
             if ((pm_lo | pm_hi) == 0u) break;
@@ -562,6 +574,7 @@ static cudaError_t launch_p(const ReplayArgs& a, bool bulk, bool lit, cudaStream
   return bulk ? launch_t<POLICY, true, 0, false>(a, stream) : launch_t<POLICY, false, 0, false>(a, stream);
 }
 
+#undef WSTORE
 }  // namespace wpt
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream) {
