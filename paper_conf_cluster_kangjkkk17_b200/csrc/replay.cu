@@ -119,6 +119,18 @@ __device__ __forceinline__ uint32_t redux_max(uint32_t v) {
     if (lane == 0) (lhs) = wstore_v_;     \
     __syncwarp();                         \
   } while (0)
+// two writes with no read of either location between them: one sync pair
+#define WSTORE2(l1, v1, l2, v2)           \
+  do {                                    \
+    const auto wstore_v1_ = (v1);         \
+    const auto wstore_v2_ = (v2);         \
+    __syncwarp();                         \
+    if (lane == 0) {                      \
+      (l1) = wstore_v1_;                  \
+      (l2) = wstore_v2_;                  \
+    }                                     \
+    __syncwarp();                         \
+  } while (0)
 
 // NF: compile-time container count (64) or 0 = runtime p.n.
 // LIT: the literal re-select-on-every-release reading R1-LIT (NEXT-1).
@@ -269,8 +281,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             target = c; a_tg = g;
           }
           const uint32_t d1 = cx[c].x;
-          WSTORE(cx[c], make_uint2(0u, adm));
-          WSTORE(cs[c], make_uint4(ust, s.y, d1, L));
+          WSTORE2(cx[c], make_uint2(0u, adm), cs[c], make_uint4(ust, s.y, d1, L));
           nk = ((t + s.z) << 6) | c;
         } else {
           const uint32_t cw = s.y;
@@ -289,12 +300,11 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
             } else {  // pause: reply withheld
               ust |= kPaused;
               const uint32_t wv = cx[c].x - t;
-              WSTORE(cx[c], make_uint2(wv, POLICY == CONVGPU_RECENT_FIT ? seq : kKeyNone));
+              WSTORE2(cx[c], make_uint2(wv, POLICY == CONVGPU_RECENT_FIT ? seq : kKeyNone), cs[c].x, ust);
               ++seq;
               if (c < 32) pm_lo |= 1u << c; else pm_hi |= 1u << (c - 32);
               adv = false;
               disp = LIT || (target == kTargetNone);
-              WSTORE(cs[c].x, ust);
             }
           } else if (kind == CONVGPU_OP_FREE) {  // P:110, R11
             if (r > used) { flags |= CONVGPU_FLAG_INVALID_FREE; break; }
@@ -424,8 +434,8 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
                 }
               }
               if (a_tg == Lt) {  // fully guaranteed: admit, cascade leftover
-                WSTORE(cx[tg].y, (t << 6) | rank); ++rank;
-                WSTORE(cs[tg], make_uint4(ut | kAdmitted, st.y, st.z, Lt));
+                WSTORE2(cx[tg].y, (t << 6) | rank, cs[tg], make_uint4(ut | kAdmitted, st.y, st.z, Lt));
+                ++rank;
                 target = kTargetNone;
                 a_tg = 0;
                 continue;
@@ -574,6 +584,7 @@ static cudaError_t launch_p(const ReplayArgs& a, bool bulk, bool lit, cudaStream
   return bulk ? launch_t<POLICY, true, 0, false>(a, stream) : launch_t<POLICY, false, 0, false>(a, stream);
 }
 
+#undef WSTORE2
 #undef WSTORE
 }  // namespace wpt
 
