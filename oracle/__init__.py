@@ -87,34 +87,51 @@ API_DTYPE = np.dtype([("api", np.uint32), ("a0", np.uint32), ("a1", np.uint32), 
 _lib = None
 
 
+def build_fault(fault: int, out_dir: str) -> str:
+    """TEST-ONLY: compile the oracle with -DORC_FAULT=<fault> (one planted bug,
+    see oracle.c) into out_dir, so tests can show the invariant checker fires."""
+    so = os.path.join(out_dir, f"liboracle_fault{fault}.so")
+    subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-fPIC", "-shared",
+                           f"-DORC_FAULT={int(fault)}", "-o", so] + _SRC)
+    return so
+
+
+def load(path: str):
+    """ctypes handle with the oracle's prototypes declared (lib() or a fault build)."""
+    return _declare(C.CDLL(path))
+
+
 def lib():
     global _lib
     if _lib is None:
         build()
-        L = C.CDLL(_SO)
-        u32p, u64p, u8p = C.POINTER(C.c_uint32), C.POINTER(C.c_uint64), C.POINTER(C.c_uint8)
-        L.orc_philox4x32_10.argtypes = [u32p, u32p, u32p]
-        L.orc_mix64.argtypes = [C.c_uint64]
-        L.orc_mix64.restype = C.c_uint64
-        L.orc_replay.argtypes = [C.POINTER(_Trace), C.c_uint32, C.c_int, C.c_uint64,
-                                 C.c_uint64, C.c_uint32, C.c_int, C.POINTER(_Result)]
-        L.orc_generate.argtypes = [C.POINTER(_Gen), C.c_uint64, u32p, u32p, u32p, u32p]
-        L.orc_replay_range.argtypes = [C.POINTER(_Gen), C.c_uint32, C.c_int, C.c_uint64,
-                                       C.c_uint32, C.c_uint64, C.c_uint64, C.c_int,
-                                       C.POINTER(Stats), u32p, u64p, u32p, u32p, u8p,
-                                       u32p, u32p]
-        L.orc_replay_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, u32p, u32p,
-                                       u32p, u32p, C.c_uint32, C.c_int, C.c_uint64,
-                                       C.c_uint64, C.c_uint32, C.c_int, C.POINTER(Stats),
-                                       u32p, u64p, u32p, u32p, u8p, u32p, u32p]
-        L.orc_wrap_bytes.argtypes = [C.POINTER(ApiOp), C.c_uint32]
-        L.orc_wrap_bytes.restype = C.c_uint64
-        L.orc_wrap_mib.argtypes = [C.c_uint64]
-        L.orc_wrap_mib.restype = C.c_uint32
-        L.orc_wrap_program.argtypes = [C.POINTER(ApiOp), C.c_uint32, C.c_uint32, u32p]
-        L.orc_wrap_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, C.c_void_p, C.c_uint32, u32p]
-        _lib = L
+        _lib = _declare(C.CDLL(_SO))
     return _lib
+
+
+def _declare(L):
+    u32p, u64p, u8p = C.POINTER(C.c_uint32), C.POINTER(C.c_uint64), C.POINTER(C.c_uint8)
+    L.orc_philox4x32_10.argtypes = [u32p, u32p, u32p]
+    L.orc_mix64.argtypes = [C.c_uint64]
+    L.orc_mix64.restype = C.c_uint64
+    L.orc_replay.argtypes = [C.POINTER(_Trace), C.c_uint32, C.c_int, C.c_uint64,
+                             C.c_uint64, C.c_uint32, C.c_int, C.POINTER(_Result)]
+    L.orc_generate.argtypes = [C.POINTER(_Gen), C.c_uint64, u32p, u32p, u32p, u32p]
+    L.orc_replay_range.argtypes = [C.POINTER(_Gen), C.c_uint32, C.c_int, C.c_uint64,
+                                   C.c_uint32, C.c_uint64, C.c_uint64, C.c_int,
+                                   C.POINTER(Stats), u32p, u64p, u32p, u32p, u8p,
+                                   u32p, u32p]
+    L.orc_replay_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, u32p, u32p,
+                                   u32p, u32p, C.c_uint32, C.c_int, C.c_uint64,
+                                   C.c_uint64, C.c_uint32, C.c_int, C.POINTER(Stats),
+                                   u32p, u64p, u32p, u32p, u8p, u32p, u32p]
+    L.orc_wrap_bytes.argtypes = [C.POINTER(ApiOp), C.c_uint32]
+    L.orc_wrap_bytes.restype = C.c_uint64
+    L.orc_wrap_mib.argtypes = [C.c_uint64]
+    L.orc_wrap_mib.restype = C.c_uint32
+    L.orc_wrap_program.argtypes = [C.POINTER(ApiOp), C.c_uint32, C.c_uint32, u32p]
+    L.orc_wrap_batch.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, C.c_void_p, C.c_uint32, u32p]
+    return L
 
 
 def _p(a, ct=C.c_uint32):
@@ -215,14 +232,15 @@ def _pack(o, st):
 
 
 def replay_range(w, policy, tid_lo: int, tid_hi: int, full: bool = False,
-                 check: bool = False, rand_seed=None):
-    """Generate + replay global trace ids [tid_lo, tid_hi) of workload w."""
+                 check: bool = False, rand_seed=None, L=None):
+    """Generate + replay global trace ids [tid_lo, tid_hi) of workload w
+    (L: another oracle build from load(), e.g. a fault build; default lib())."""
     g = w.gen
     count = tid_hi - tid_lo
     o = _outputs(count, g.n, full)
     st = Stats()
     seed = w.rand_seed if rand_seed is None else rand_seed
-    rc = lib().orc_replay_range(C.byref(gen_struct(g)), w.cap, _pol(policy), seed, w.ovh,
+    rc = (L or lib()).orc_replay_range(C.byref(gen_struct(g)), w.cap, _pol(policy), seed, w.ovh,
                                 tid_lo, tid_hi, 1 if check else 0, C.byref(st),
                                 _p(o["sum_u32x4"]), _p(o["sum_u64x2"], C.c_uint64),
                                 _p(o["cnt_u32x2"]), _p(o["admit_tick"]),
@@ -232,13 +250,13 @@ def replay_range(w, policy, tid_lo: int, tid_hi: int, full: bool = False,
     return res
 
 
-def replay_batch(b, cap, policy, tid_base=0, rand_seed=0, ovh=0, check=False, full=True):
-    """Replay a workloads.Batch (numpy) with the oracle."""
+def replay_batch(b, cap, policy, tid_base=0, rand_seed=0, ovh=0, check=False, full=True, L=None):
+    """Replay a workloads.Batch (numpy) with the oracle (L: see replay_range)."""
     count, n, K = b.count, b.n, b.K
     o = _outputs(count, n, full)
     st = Stats()
     arrs = [np.ascontiguousarray(x, np.uint32) for x in (b.arrival, b.limit, b.delta, b.arg)]
-    rc = lib().orc_replay_batch(n, K, count, *[_p(x) for x in arrs], cap, _pol(policy),
+    rc = (L or lib()).orc_replay_batch(n, K, count, *[_p(x) for x in arrs], cap, _pol(policy),
                                 tid_base, rand_seed, ovh, 1 if check else 0, C.byref(st),
                                 _p(o["sum_u32x4"]), _p(o["sum_u64x2"], C.c_uint64),
                                 _p(o["cnt_u32x2"]), _p(o["admit_tick"]),

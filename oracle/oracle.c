@@ -23,6 +23,15 @@
 
 #define TICK_LIMIT (1ull << 26) /* R19: packed (tick, index) horizon */
 
+/* Fault injection, TEST-ONLY (tests/test_oracle_faults.py): a build with
+ * -DORC_FAULT=<n> plants one deliberate bug so the tests can show that the
+ * invariant checker fires on it.  The normal build defines nothing, and then
+ * FAULT(n) is 0 everywhere, so the replay below is unchanged. */
+#ifndef ORC_FAULT
+#define ORC_FAULT 0
+#endif
+#define FAULT(n) (ORC_FAULT == (n))
+
 /* ------------------------------------------------------------------ */
 /* Philox4x32-10 (Salmon et al., SC'11; Random123 constants).  Used for
  * Random-Fit selection (R6) and the synthetic workload (DESIGN.md recipe). */
@@ -133,7 +142,7 @@ static void ev_arrive(sim_t *s, int c, uint32_t t) {
   if (s->lit || s->target < 0) g = (L < s->free_mem) ? L : s->free_mem;
   x->a = g;
   s->free_mem -= g;
-  if (g == L)
+  if (g == L || (FAULT(6) && g > 0))
     admit(s, c, t);
   else if (g > 0 && !s->lit)
     s->target = c;
@@ -149,7 +158,7 @@ static void ev_alloc(sim_t *s, int c, uint32_t t, uint32_t r) {
   if (need > L_of(s, c)) {            /* over the declared limit: reject (R10) */
     s->n_rejected++;
     advance(s, c, t);
-  } else if (need <= x->a) {          /* within the assigned memory: grant */
+  } else if (need <= x->a || FAULT(3)) { /* within the assigned memory: grant */
     x->used = (uint32_t)need;
     x->first_done = 1;
     advance(s, c, t);
@@ -179,12 +188,12 @@ static void ev_free(sim_t *s, int c, uint32_t t, uint32_t r) {
  * to the scheduler, which can assign it to other containers). */
 static void ev_finish(sim_t *s, int c, uint32_t t) {
   cont_t *x = &s->c[c];
-  s->free_mem += x->a;
+  if (!FAULT(1)) s->free_mem += x->a;
   x->a = 0;
   x->used = 0;
   x->st = ST_DONE;
   x->finish = t;
-  if (s->target == c) s->target = -1; /* R20: target left before it was full */
+  if (s->target == c && !FAULT(5)) s->target = -1; /* R20: target left before it was full */
 }
 
 /* SELECT among paused containers. */
@@ -301,14 +310,14 @@ static void dispatch(sim_t *s, uint32_t t) {
       cont_t *x = &s->c[tg];
       uint32_t L = L_of(s, tg);
       uint32_t room = L - x->a;
-      uint32_t g = (s->free_mem < room) ? s->free_mem : room;
+      uint32_t g = (s->free_mem < room || FAULT(2)) ? s->free_mem : room;
       x->a += g;
       s->free_mem -= g;
       if (x->paused && (uint64_t)x->used + x->pending <= x->a) { /* RESUME */
         x->used += x->pending;
         x->first_done = 1;
         x->paused = 0;
-        x->wait += t - x->susp_tick;
+        if (!FAULT(4)) x->wait += t - x->susp_tick;
         advance(s, tg, t);
       }
       if (x->a == L) {

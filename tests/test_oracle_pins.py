@@ -373,3 +373,27 @@ def test_literal_reading_invariants_and_deadlock_rate(orc, policy):
     assert sticky["rc"] == 0 and lit["rc"] == 0
     assert sticky["stats"]["flag_count"][0] == 0
     assert lit["stats"]["flag_count"][1] == 0  # never overcommits
+
+
+@pytest.mark.parametrize("case", range(4))
+def test_generator_exact_values(orc, case):
+    """orc_generate against values derived BY HAND from the recipe
+    (tests/golden/generator_cases.json 'work'): the per-op split s1 = e/2,
+    s2 = e - s1, d1 = dur/4, d2 = dur/2, d3 = dur - d1 - d2, e = max(L - ovh, 0),
+    the jitter term, the class offset, 64-bit trace ids and the K = 2
+    program.  Swapping d1/d2 or s1/s2, dropping ovh or the jitter each fail
+    one of the four cases."""
+    from oracle import bruteforce
+    cs = golden("generator_cases.json")["cases"][case]
+    g = W.GenParams(**{k: (tuple(v) if k == "class_mib" else v) for k, v in cs["gen"].items()})
+    tid, c = cs["tid"], cs["c"]
+    # the two Philox words the derivation starts from (Philox is KAT-pinned)
+    x = bruteforce.philox4x32_10([tid & 0xFFFFFFFF, tid >> 32, c, 0],
+                                 [g.gen_seed & 0xFFFFFFFF, g.gen_seed >> 32])
+    assert x[0] == h(cs["x0"]) and x[1] == h(cs["x1"])
+    a, L, d, arg = orc.generate(g, tid)
+    assert int(a[c]) == cs["arrival"]
+    assert int(L[c]) == cs["limit"]
+    assert [int(v) for v in d[:, c]] == cs["delta"]
+    assert [int(v) >> 30 for v in arg[:, c]] == cs["kind"]
+    assert [int(v) & 0x3FFFFFFF for v in arg[:, c]] == cs["size"]
