@@ -5,14 +5,24 @@ GPU-memory scheduler (BASELINE.json metric), one JSON line on rank 0.
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
 Workload (N=1): BASELINE.json configs[2] — 10^6 traces x 64 containers, 2x
-oversubscription of a 180 GiB GPU (workloads.CONFIGS["c2"]).  Under torchrun
-(N>1) every rank replays its own 10^6-trace shard of the global id space
-(weak scaling; config [3]'s sharding) and the per-policy statistics are
-all-reduced over NCCL each step.  A "step" = the whole hot path over the
-batch: replay under FIFO, Best-Fit, Recent-Fit and Random-Fit (4 launches of
-the replay kernel, full per-container outputs + summaries + statistics).
-Inputs (2.56 GB per rank) are resident in HBM before the timed region and are
-larger than the 126 MB L2, so no flush is needed between steps.
+oversubscription of a 180 GiB GPU (workloads.CONFIGS["c2"]).  Rank r replays
+global ids [r * 2^20, r * 2^20 + 10^6), so that after the timed steps the
+replayed ids plus an untimed tail are exactly 2^20-trace range r of the
+oracle's golden file (tests/golden/c3_range_digests.json): every bench run
+checks every rank's per-policy digest sum, events, waits, selections and
+makespans against the oracle and reports it under "parity" (exit 3 on a
+mismatch).  Under torchrun (N>1) this is weak scaling; the per-policy
+statistics are all-reduced over NCCL each step and the per-range rows once
+after the timed steps.  A "step" = the whole hot path over the batch: replay
+under FIFO, Best-Fit, Recent-Fit and Random-Fit (4 launches of the replay
+kernel, full per-container outputs + summaries + statistics).  Inputs (2.56
+GB per rank) are resident in HBM before the timed region and are larger than
+the 126 MB L2, so no flush is needed between steps.  `value` uses the median
+step time (median of >= 5 repetitions).
+
+`--workload c3`: BASELINE configs[3] — 10^8 traces sharded [r*N/G, (r+1)*N/G),
+chunked generate -> replay on every rank, all 96 golden ranges x 4 policies
+checked after an NCCL all-reduce of the range digests (run_c3).
 
 `--impl reference` times the C oracle (test infrastructure, the only
 reference this paper-only task has) on the host cores on a bounded sample of
@@ -29,6 +39,8 @@ import sys
 import threading
 import time
 
+import numpy as np
+
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
@@ -44,13 +56,15 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="c2", choices=["c1", "c2", "mimic"])
+    ap.add_argument("--workload", default="c2", choices=["c1", "c2", "c3", "mimic"])
     ap.add_argument("--traces", type=int, default=None, help="traces per GPU (default: config)")
     ap.add_argument("--outputs", default="full", choices=["full", "summary"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane", "lane16"])
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--e2e-chunk", type=int, default=1 << 15, help="traces per host-path chunk")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-check", action="store_true", help="skip the golden-range parity check")
+    ap.add_argument("--c3-chunk", type=int, default=4 << 20, help="traces per chunk (config [3])")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=32768, help="traces per policy (cpu leg)")
     ap.add_argument("--ref-sample", type=int, default=4096, help="traces per policy per step (reference arm)")
@@ -184,7 +198,7 @@ def run_reference(args, rank, world):
                    "ops_per_container": w.gen.K, "capacity_mib": w.cap,
                    "policies": list(POLICIES)},
         "cpu_baseline": {"value": value, "unit": "events/s", "cores": C, "kind": "oracle",
-                         "sample": sample},
+                         "cpu_model": cpu_model(), "sample": sample},
         "e2e": {"value": value, "unit": "events/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -199,6 +213,7 @@ def cpu_baseline(w, sample):
     ev1, dt1 = oracle_run(w, sample, 1)
     evc, dtc = oracle_run(w, sample * C // 2, C)
     return {"value": evc / dtc, "unit": "events/s", "cores": C, "kind": "oracle",
+            "cpu_model": cpu_model(),
             "sample": f"{sample * C // 2} traces x {len(POLICIES)} policies of {w.name} "
                       f"(ids 0..{sample * C // 2 - 1}), {C} threads of the single-threaded C "
                       f"oracle on disjoint id ranges, {dtc:.1f} s",
@@ -228,6 +243,70 @@ def ncu_summary(workload, traces):
     return {}
 
 
+# ------------------------------------------------------------------ parity
+GOLDEN = os.path.join(ROOT, "tests", "golden", "c3_range_digests.json")
+RANGE = 1 << 20  # traces per golden range
+RANGE_FIELDS = ("digest_sum", "events", "sum_wait", "n_select", "sum_makespan", "traces")
+
+
+def load_golden(w):
+    """Per-2^20-trace-range results of the C oracle for the config [2] / [3]
+    generator (tests/golden/c3_range_digests.json, written by
+    scripts/c3_oracle_digests.py from oracle/ only; read here as data — no
+    oracle code runs).  None if `w` is another workload."""
+    c3 = W.CONFIGS["c3"]
+    if (w.gen, w.cap, w.ovh, w.rand_seed) != (c3.gen, c3.cap, c3.ovh, c3.rand_seed):
+        return None
+    try:
+        with open(GOLDEN) as f:
+            g = json.load(f)
+    except OSError:
+        return None
+    return g if g.get("range_size") == RANGE else None
+
+
+def golden_row(g, policy, r):
+    e = g["policies"].get(policy, {}).get(str(r))
+    if e is None:
+        return None
+    return [int(e["digest"], 16), e["events"], e["sum_wait"], e["n_select"], e["sum_makespan"],
+            e["traces"]]
+
+
+def s64(v: int) -> int:
+    v &= (1 << 64) - 1
+    return v - (1 << 64) if v >> 63 else v
+
+
+def stats_row(st) -> list:
+    return [st[f] for f in RANGE_FIELDS]
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def max_over_ranks_vec(xs, device, world):
+    """Element-wise max over ranks of a list of floats (per-step times)."""
+    if world == 1:
+        return list(xs)
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor(xs, dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return [float(v) for v in t.cpu()]
+
+
+SPEC_HBM_GBS = 8000.0  # B200 HBM3e nominal (B200_PROFILING.md), for the "% of spec" figure
+
+
 def run_ours(args, rank, local_rank, world):
     import torch
     import torch.distributed as dist
@@ -248,10 +327,18 @@ def run_ours(args, rank, local_rank, world):
         else:
             dist.init_process_group(backend)
     cg.lib()
+    if args.workload == "c3":
+        return run_c3(args, rank, world, dev, cg, cgd)
     w = W.CONFIGS[args.workload]
-    Nr = args.traces or (w.n_traces if args.workload != "c3" else w.n_traces // world)
+    Nr = args.traces or w.n_traces
     n, K = w.gen.n, w.gen.K
-    base = rank * Nr  # rank r owns global ids [r*Nr, (r+1)*Nr)
+    golden = None if args.no_check else load_golden(w)
+    if golden is not None and Nr > RANGE:
+        golden = None
+    # rank r owns global ids [base, base + Nr).  With the config [2] / [3]
+    # generator the shard starts at a golden range (base = r * 2^20), so the
+    # replayed ids plus an untimed tail are exactly oracle range r.
+    base = rank * (RANGE if golden is not None else Nr)
     stream = torch.cuda.current_stream()
 
     # a0: generation (timed separately, not part of events/s; the first call
@@ -270,6 +357,7 @@ def run_ours(args, rank, local_rank, world):
     stats = {p: torch.zeros(nsteps, 12, dtype=torch.int64, device=dev) for p in POLICIES}
     ev_s = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
     ev_e = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
+    step_ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
 
     def step(s, timed_idx=None):
         for p in POLICIES:
@@ -295,18 +383,19 @@ def run_ours(args, rank, local_rank, world):
         phys = int(vis.split(",")[dev.index]) if vis else dev.index
         sampler = ClockSampler(phys)
         sampler.start()
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
-    t_start.record(stream)
+    step_ev[0].record(stream)
     for k in range(args.steps):
         step(args.warmup + k, k)
-    t_end.record(stream)
+        step_ev[k + 1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clocks = sampler.stop() if sampler else None
-    ms_local = t_start.elapsed_time(t_end)
-    ms = cgd.max_over_ranks(ms_local, dev)
+    step_ms = max_over_ranks_vec([step_ev[k].elapsed_time(step_ev[k + 1]) for k in range(args.steps)],
+                                 dev, world)
+    ms_total = cgd.max_over_ranks(step_ev[0].elapsed_time(step_ev[-1]), dev)
+    ms_med = statistics.median(step_ms)
 
     per_trace_events = n * (1 + K)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
@@ -316,23 +405,71 @@ def run_ours(args, rank, local_rank, world):
             return args.kernel
         if Nr < sms * 40:
             return "warp"
-        return "lane16" if (full and n == 64 and K == 4) else "lane"
+        return "lane16" if (n == 64 and K == 4) else "lane"
     launches_per_replay = {p: 2 if kernel_of(p) == "lane16" else 1 for p in POLICIES}
-    kernel_used = ",".join(sorted({kernel_of(p) for p in POLICIES}))
     # correctness of the timed work: every timed launch replayed every trace
     last = args.warmup + args.steps - 1
     checks = {}
     for p in POLICIES:
         st = cg.stats_dict(stats[p][last].cpu().numpy().view(cg.STATS_DTYPE)[0])
-        exp_ev = Nr * per_trace_events * (world if world > 1 else 1)
+        exp_ev = Nr * per_trace_events * world
         assert st["events"] == exp_ev, (p, st["events"], exp_ev)
         assert st["flag_count"] == [0] * 8, (p, st["flag_count"])
         checks[p] = st
-    launch_ms = {p: statistics.mean(ev_s[p][k].elapsed_time(ev_e[p][k]) for k in range(args.steps))
+    launch_ms = {p: statistics.median(ev_s[p][k].elapsed_time(ev_e[p][k]) for k in range(args.steps))
                  for p in POLICIES}
 
-    events_total = world * args.steps * len(POLICIES) * Nr * per_trace_events
-    value = events_total / (ms / 1e3)
+    events_per_step = world * len(POLICIES) * Nr * per_trace_events
+    value = events_per_step / (ms_med / 1e3)
+
+    # parity of the timed work against the oracle (after the timed region):
+    # rank r's timed ids + the untimed tail [base + Nr, base + 2^20) form
+    # golden range r; per-range rows are SUM-all-reduced (disjoint rows) and
+    # rank 0 compares every rank's row with the oracle's
+    parity = None
+    if golden is not None and not args.profile:
+        nt = RANGE - Nr
+        rows = {p: torch.zeros(world, len(RANGE_FIELDS), dtype=torch.int64, device=dev) for p in POLICIES}
+        tail_st = {p: None for p in POLICIES}
+        if nt:
+            ttr = cg.generate(w.gen, base + Nr, nt, device=dev)
+            for p in POLICIES:
+                o = cg.alloc_out(nt, n, device=dev, full=False, summary=False)
+                cg.replay(ttr, w.cap, p, o, rand_seed=w.rand_seed, ovh=w.ovh, stream=stream,
+                          kernel=args.kernel)
+                tail_st[p] = o.stats
+            torch.cuda.synchronize()
+        # rank r's own row: under N > 1 the timed records were all-reduced in
+        # place, so replay rank r's timed ids once more (stats only, same
+        # kernel, untimed); at N = 1 that record must equal the timed one
+        for p in POLICIES:
+            o = cg.alloc_out(Nr, n, device=dev, full=False, summary=False)
+            cg.replay(tr, w.cap, p, o, rand_seed=w.rand_seed, ovh=w.ovh, stream=stream,
+                      kernel=args.kernel)
+            torch.cuda.synchronize()
+            own = cg.stats_dict(o.stats_np())
+            if world == 1:  # the timed launch's own record must agree
+                assert stats_row(own) == stats_row(checks[p]), p
+            row = stats_row(own)
+            if tail_st[p] is not None:
+                t = cg.stats_dict(tail_st[p].cpu().numpy().view(cg.STATS_DTYPE)[0])
+                row = [a + b for a, b in zip(row, stats_row(t))]
+            rows[p][rank] = torch.tensor([s64(v) for v in row], dtype=torch.int64)
+            cgd.reduce_range_digests(rows[p])
+        bad = []
+        for p in POLICIES:
+            got = rows[p].cpu().numpy().astype(np.int64).view(np.uint64)
+            for r in range(world):
+                want = golden_row(golden, p, r)
+                have = [int(v) for v in got[r]]
+                if want is None or have != want:
+                    bad.append({"policy": p, "range": r, "have": have, "want": want})
+        parity = {"ranges": world * len(POLICIES), "equal": not bad,
+                  "fields": list(RANGE_FIELDS), "range_size": RANGE,
+                  "traces_timed_per_rank": Nr, "tail_traces_per_rank": nt,
+                  "source": "tests/golden/c3_range_digests.json (C oracle, scripts/c3_oracle_digests.py)"}
+        if bad:
+            parity["mismatches"] = bad[:8]
 
     # roofline of the replay kernel (dominant kernel)
     in_b = n * (2 + 2 * K) * 4
@@ -344,6 +481,7 @@ def run_ours(args, rank, local_rank, world):
     ncu = ncu_summary(w.name, Nr)
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": ncu.get("dram_bytes_per_launch"),
+                "frac_of_spec": achieved / SPEC_HBM_GBS, "spec_peak": SPEC_HBM_GBS,
                 "ncu_limiter": ncu.get("limiter"), "ncu_source": ncu.get("source"),
                 "kernel": "replay kernels: " + ", ".join(
                     f"{p}={kernel_of(p)}" for p in POLICIES),
@@ -381,13 +519,17 @@ def run_ours(args, rank, local_rank, world):
     if rank == 0:
         result = {
             "metric": METRIC, "value": value, "unit": "events/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_med,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
+            "timing": {"value_from": "median over steps of the per-step time (CUDA events on the "
+                                     "launching stream, max over ranks)",
+                       "step_ms": step_ms, "mean_ms_per_step": ms_total / args.steps,
+                       "value_from_mean": events_per_step * args.steps / (ms_total / 1e3)},
             "config": {"workload": w.name + " (BASELINE configs[%s])" % {"c1": 1, "c2": 2}.get(args.workload, "-"),
                        "traces_per_gpu": Nr, "containers": n, "ops_per_container": K,
                        "capacity_mib": w.cap, "policies": list(POLICIES), "outputs": args.outputs,
-                       "global_trace_ids": f"[r*{Nr}, (r+1)*{Nr}) per rank r",
+                       "global_trace_ids": f"[r*{RANGE if golden is not None else Nr}, +{Nr}) per rank r",
                        "l2": "inputs %.2f GB per rank > 126 MB L2; no flush" % (Nr * in_b / 1e9),
                        "parallelism": f"dp{world} (trace-id shards, NCCL stats all-reduce)"},
             "per_policy": {p: {"events_per_s": Nr * per_trace_events * world / (launch_ms[p] / 1e3),
@@ -395,6 +537,7 @@ def run_ours(args, rank, local_rank, world):
                                "digest_sum": "%016x" % (checks[p]["digest_sum"] & (2**64 - 1)),
                                "sum_wait": checks[p]["sum_wait"],
                                "sum_makespan": checks[p]["sum_makespan"]} for p in POLICIES},
+            "parity": parity,
             "gen_ms": gen_ms,
             "gen_write_gbs": Nr * in_b / (gen_ms / 1e3) / 1e9,
             "roofline": roofline,
@@ -412,37 +555,41 @@ def run_ours(args, rank, local_rank, world):
             h.copy_(t)
         del outs
         torch.cuda.empty_cache()
-        import numpy as np
         hsum_t = torch.empty(len(POLICIES) * Nr * 5, dtype=torch.int64, pin_memory=True)
         hsum = hsum_t.numpy().view(cg.SUMMARY_DTYPE).reshape(len(POLICIES), Nr)
         ws = torch.empty(cg.host_workspace_bytes(n, K, chunk, len(POLICIES)), dtype=torch.uint8,
                          device=dev)
         cg.replay_host(*hbuf, w.cap, POLICIES, trace_id_base=base, rand_seed=w.rand_seed,
                        ovh=w.ovh, chunk=chunk, summary=hsum, workspace=ws, stream=stream)
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        e0.record(stream)
+        e2e_ms = []
         for _ in range(args.e2e_steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
             st_host = cg.replay_host(*hbuf, w.cap, POLICIES, trace_id_base=base,
                                      rand_seed=w.rand_seed, ovh=w.ovh, chunk=chunk,
                                      summary=hsum, workspace=ws, stream=stream,
                                      kernel=args.kernel)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        e2e_ms = cgd.max_over_ranks(e0.elapsed_time(e1), dev)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            e2e_ms.append(e0.elapsed_time(e1))
+        e2e_ms = max_over_ranks_vec(e2e_ms, dev, world)
         for q, p in enumerate(POLICIES):
             assert int(st_host[q]["events"]) == Nr * per_trace_events
             if rank == 0 and world == 1:
                 assert "%016x" % int(st_host[q]["digest_sum"]) == result["per_policy"][p]["digest_sum"]
         if rank == 0:
             result["e2e"] = {
-                "value": world * args.e2e_steps * len(POLICIES) * Nr * per_trace_events / (e2e_ms / 1e3),
-                "unit": "events/s", "steps": args.e2e_steps,
+                "value": events_per_step / (statistics.median(e2e_ms) / 1e3),
+                "unit": "events/s", "steps": args.e2e_steps, "step_ms": e2e_ms,
                 "h2d_bytes_per_step": Nr * in_b,
                 "d2h_bytes_per_step": len(POLICIES) * (Nr * 40 + 96),
                 "api": "convgpu_replay_host (pinned host buffers, %d-trace chunks, copy/compute overlap)" % chunk,
+                "outputs": "per-trace 40-B summaries (all fields + digest) and the statistics record "
+                           "per policy, read back to host each step; per-container outputs are not "
+                           "copied back (the device-timed `value` writes them to HBM)",
             }
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile:
         result["cpu_baseline"] = cpu_baseline(w, args.cpu_sample)
@@ -451,6 +598,155 @@ def run_ours(args, rank, local_rank, world):
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+    if parity is not None and not parity["equal"]:
+        sys.exit(3)
+
+
+def run_c3(args, rank, world, dev, cg, cgd):
+    """BASELINE config [3]: 10^8 traces (config [2] generator) sharded over the
+    ranks as contiguous global-id ranges [r*N/G, (r+1)*N/G); each rank cycles
+    generate -> replay (4 policies, summary-free: statistics + per-2^20-range
+    digests through the admission scratch on the compact kernel) over chunks
+    of its range.  After the timed steps the per-range digests and statistics
+    are all-reduced (NCCL over NVLink; the only exchange) and rank 0 checks
+    all 96 ranges x 4 policies against the oracle's golden digests."""
+    import torch
+    import torch.distributed as dist
+
+    w = W.CONFIGS["c3"]
+    total = args.traces or w.n_traces
+    lo, hi = cgd.shard_range(total, rank, world)
+    cnt = hi - lo
+    n, K = w.gen.n, w.gen.K
+    chunk = min(args.c3_chunk, max(cnt, 1))
+    nr = (total + RANGE - 1) // RANGE
+    stream = torch.cuda.current_stream()
+    tr = cg.empty_traces(chunk, n, K, device=dev)
+    scratch = torch.empty(chunk, n, dtype=torch.int32, device=dev)
+    outs = {}
+    for p in POLICIES:
+        o = cg.alloc_out(chunk, n, device=dev, full=False, summary=False, range_count=nr,
+                         range_size=RANGE, scratch=False)
+        o.admit_scratch = scratch
+        outs[p] = o
+    nchunks = (cnt + chunk - 1) // chunk
+    rep_ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in POLICIES] for _ in range(nchunks)]
+    gen_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(nchunks)]
+
+    def step(timed):
+        for p in POLICIES:
+            outs[p].stats.zero_()
+            outs[p].range_digest.zero_()
+        for j in range(nchunks):
+            a = lo + j * chunk
+            c = min(chunk, hi - a)
+            sub = cg.Traces(tr.arrival[:c], tr.limit[:c], tr.op_delta[:c], tr.op_arg[:c])
+            if timed:
+                gen_ev[j][0].record(stream)
+            cg.generate(w.gen, a, c, out=sub, stream=stream)
+            if timed:
+                gen_ev[j][1].record(stream)
+            for q, p in enumerate(POLICIES):
+                if timed:
+                    rep_ev[j][q][0].record(stream)
+                cg.replay(sub, w.cap, p, outs[p], rand_seed=w.rand_seed, ovh=w.ovh, stream=stream,
+                          kernel=args.kernel)
+                if timed:
+                    rep_ev[j][q][1].record(stream)
+
+    for _ in range(args.warmup):
+        step(False)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+    phys = int(vis.split(",")[dev.index]) if vis else dev.index
+    sampler = None if args.profile else ClockSampler(phys)
+    if sampler:
+        sampler.start()
+    step_ms, rep_ms, gen_ms = [], [], []
+    for _ in range(args.steps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step(True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        step_ms.append(e0.elapsed_time(e1))
+        rep_ms.append(sum(a.elapsed_time(b) for row in rep_ev for a, b in row))
+        gen_ms.append(sum(a.elapsed_time(b) for a, b in gen_ev))
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop() if sampler else None
+    step_ms = max_over_ranks_vec(step_ms, dev, world)
+    rep_ms = max_over_ranks_vec(rep_ms, dev, world)
+    # the one exchange: statistics + per-range digests of the last step
+    for p in POLICIES:
+        cgd.reduce_stats(outs[p].stats)
+        cgd.reduce_range_digests(outs[p].range_digest)
+    torch.cuda.synchronize()
+    per_trace_events = n * (1 + K)
+    events_per_step = total * per_trace_events * len(POLICIES)
+    if rank == 0:
+        g = load_golden(w)
+        bad, checked = [], 0
+        per_policy = {}
+        for p in POLICIES:
+            st = cg.stats_dict(outs[p].stats_np())
+            rd = outs[p].range_digest.cpu().numpy().view(np.uint64)
+            tot = [0] * len(RANGE_FIELDS)
+            for r in range(nr):
+                want = golden_row(g, p, r) if g else None
+                if want is None:
+                    bad.append({"policy": p, "range": r, "missing": True})
+                    continue
+                checked += 1
+                if int(rd[r]) != want[0]:
+                    bad.append({"policy": p, "range": r, "have": "%016x" % int(rd[r]),
+                                "want": "%016x" % want[0]})
+                tot = [a + b for a, b in zip(tot, want)]
+            tot[0] &= (1 << 64) - 1
+            have = stats_row(st)
+            have[0] &= (1 << 64) - 1
+            if total == w.n_traces and have != tot:
+                bad.append({"policy": p, "totals": True, "have": have, "want": tot})
+            if st["flag_count"] != [0] * 8:
+                bad.append({"policy": p, "flags": st["flag_count"]})
+            per_policy[p] = {"digest_sum": "%016x" % have[0], "events": st["events"],
+                             "sum_wait": st["sum_wait"], "n_select": st["n_select"]}
+        ms_med = statistics.median(step_ms)
+        result = {
+            "metric": METRIC, "value": events_per_step / (ms_med / 1e3), "unit": "events/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_med,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": w.name + " (BASELINE configs[3])", "traces_total": total,
+                       "traces_per_gpu": cnt, "chunk_traces": chunk, "containers": n,
+                       "ops_per_container": K, "capacity_mib": w.cap, "policies": list(POLICIES),
+                       "outputs": "statistics + per-2^20-range digests (summary-free)",
+                       "global_trace_ids": "[r*N/G, (r+1)*N/G) per rank r",
+                       "step": "generate + replay x 4 policies per chunk, every chunk of the shard",
+                       "l2": "inputs %.1f GB per chunk > 126 MB L2; no flush" % (chunk * n * 40 / 1e9),
+                       "parallelism": f"dp{world} (trace-id shards, NCCL all-reduce of stats + range digests)"},
+            "timing": {"value_from": "median step time incl. on-device generation (max over ranks)",
+                       "step_ms": step_ms, "replay_ms": rep_ms,
+                       "replay_only_events_per_s": events_per_step / (statistics.median(rep_ms) / 1e3)},
+            "per_policy": per_policy,
+            "parity": {"ranges": checked, "equal": not bad, "range_size": RANGE,
+                       "fields": ["range digest"] + ["totals: " + ",".join(RANGE_FIELDS[1:])],
+                       "source": "tests/golden/c3_range_digests.json (C oracle, scripts/c3_oracle_digests.py)",
+                       **({"mismatches": bad[:8]} if bad else {})},
+            "gpu_launches": args.steps * nchunks * (1 + 2 * len(POLICIES)),
+            "clocks": clocks,
+        }
+        print(json.dumps(result), flush=True)
+        ok = not bad
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    if rank == 0 and not ok:  # noqa: F821 (set on rank 0 above)
+        sys.exit(3)
 
 
 def main():

@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define CONVGPU_ABI_VERSION 3
+#define CONVGPU_ABI_VERSION 4
 #define CONVGPU_MAX_CONTAINERS 64u   /* containers per trace */
 #define CONVGPU_MAX_OPS 8u           /* ops per container (K) */
 #define CONVGPU_CAPACITY_LIMIT (1u << 26) /* capacity_mib must be below this */
@@ -113,8 +113,9 @@ enum {
   CONVGPU_KERNEL_LANE_PER_TRACE = 2, /* one lane per trace, 32 traces per warp */
   CONVGPU_KERNEL_LANE_COMPACT = 3    /* one lane per trace, 16-bit packed state, up to
                                         8 warps per SM; needs n_containers = 64, n_ops = 4,
-                                        out->admit_tick != NULL (it holds admissions during
-                                        the replay) and 16-byte aligned arrays / outputs,
+                                        out->admit_tick or out->admit_scratch != NULL (it
+                                        holds admissions during the replay) and 16-byte
+                                        aligned arrays / outputs,
                                         else -EINVAL.  Traces whose limits exceed 0xFFFE
                                         MiB, deltas 0xFFFF ticks or horizon 2^25 are
                                         replayed by a second, 32-bit lane-per-trace launch.
@@ -153,6 +154,14 @@ typedef struct {
   uint64_t *range_digest;     /* optional: range_digest[gid / range_size] += digest */
   uint64_t range_size;        /* > 0 when range_digest != NULL */
   void *stream;               /* cudaStream_t */
+  /* Optional caller-owned DEVICE scratch, [n][n_containers] u32, 16-byte
+   * aligned (ABI 4).  The compact lane kernel keeps each container's
+   * admission in its slot while the trace replays (admit_tick itself serves
+   * when it is requested).  With admit_tick == NULL and this scratch given,
+   * summary- / digest- / stats-only launches still run on the compact kernel;
+   * without either, AUTO falls back to the 32-bit lane kernel.  Contents are
+   * undefined after the call; NULL allowed. */
+  uint32_t *admit_scratch;
 } convgpu_out_t;
 
 /*

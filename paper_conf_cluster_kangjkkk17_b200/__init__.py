@@ -57,7 +57,8 @@ class TracesT(C.Structure):
 class OutT(C.Structure):
     _fields_ = [("admit_tick", C.c_void_p), ("admit_rank", C.c_void_p), ("wait", C.c_void_p),
                 ("finish", C.c_void_p), ("summary", C.c_void_p), ("stats", C.c_void_p),
-                ("range_digest", C.c_void_p), ("range_size", C.c_uint64), ("stream", C.c_void_p)]
+                ("range_digest", C.c_void_p), ("range_size", C.c_uint64), ("stream", C.c_void_p),
+                ("admit_scratch", C.c_void_p)]
 
 
 class GenParamsT(C.Structure):
@@ -229,6 +230,8 @@ class ReplayOut:
     finish: Optional["torch.Tensor"] = None
     range_digest: Optional["torch.Tensor"] = None  # int64 [R]
     range_size: int = 0
+    admit_scratch: Optional["torch.Tensor"] = None  # int32 [N, n]: lets summary-only
+    #                                                  launches use the compact kernel
 
     # host views (after synchronisation)
     def summary_np(self) -> np.ndarray:
@@ -249,9 +252,16 @@ class ReplayOut:
 
 
 def alloc_out(count: int, n: int, device="cuda", full=True, summary=True, stats=True,
-              range_count: int = 0, range_size: int = 0) -> ReplayOut:
+              range_count: int = 0, range_size: int = 0, scratch: bool = None) -> ReplayOut:
+    """Device output buffers.  scratch (default: when per-container outputs are
+    not requested) adds the admission scratch of convgpu_out_t, so that
+    summary- / digest-only replays run on the compact lane kernel."""
     import torch
     o = ReplayOut()
+    if scratch is None:
+        scratch = not full
+    if scratch and not full:
+        o.admit_scratch = torch.empty(count, n, dtype=torch.int32, device=device)
     if summary:
         o.summary = torch.empty(count, 5, dtype=torch.int64, device=device)
     if stats:
@@ -276,7 +286,7 @@ def replay(traces: Traces, capacity: int, policy, out: ReplayOut, rand_seed: int
     tr = traces.struct(rand_seed, ovh, kernel)
     o = OutT(_ptr(out.admit_tick), _ptr(out.admit_rank), _ptr(out.wait), _ptr(out.finish),
              _ptr(out.summary), _ptr(out.stats), _ptr(out.range_digest), out.range_size,
-             _stream_handle(stream))
+             _stream_handle(stream), _ptr(out.admit_scratch))
     _check(lib().convgpu_replay(C.byref(tr), traces.count, capacity, _pol(policy), C.byref(o)),
            "convgpu_replay")
     return out

@@ -29,20 +29,42 @@ def _stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every translation unit to an object in parallel (the units are
+    independent: no relocatable device code), then link the shared library."""
     if not force and not _stale():
         return SO
+    from concurrent.futures import ThreadPoolExecutor
+    objdir = os.path.join(PKG, "build")
+    os.makedirs(objdir, exist_ok=True)
+
+    def compile_one(f):
+        obj = os.path.join(objdir, f.replace(".cu", ".o"))
+        cmd = [NVCC, *FLAGS, "-c", "-o", obj, os.path.join(CSRC, f)]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        return obj, cmd, r
+
+    with ThreadPoolExecutor(len(SOURCES)) as ex:
+        results = list(ex.map(compile_one, SOURCES))
     tmp = SO + ".tmp"
-    cmd = [NVCC, *FLAGS, "-shared", "-o", tmp] + [os.path.join(CSRC, f) for f in SOURCES]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+    link = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp] + \
+        [o for o, _, _ in results]
     log = os.path.join(PKG, "build.log")
+    failed = [r for _, _, r in results if r.returncode != 0]
     with open(log, "w") as f:
-        f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
+        for _, cmd, r in results:
+            f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
+    if failed:
+        sys.stderr.write("".join(r.stdout + r.stderr for r in failed))
+        raise RuntimeError(f"nvcc failed; see {log}")
+    r = subprocess.run(link, capture_output=True, text=True)
+    with open(log, "a") as f:
+        f.write(" ".join(link) + "\n" + r.stdout + r.stderr)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError(f"nvcc failed ({r.returncode}); see {log}")
+        raise RuntimeError(f"nvcc link failed ({r.returncode}); see {log}")
     os.replace(tmp, SO)
     if verbose:
-        sys.stderr.write(r.stderr)
+        sys.stderr.write("".join(r.stderr for _, _, r in results))
     return SO
 
 

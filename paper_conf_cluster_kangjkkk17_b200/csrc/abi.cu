@@ -100,8 +100,8 @@ uint32_t auto_variant(uint64_t count, int policy) {
 }
 
 cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cudaStream_t s) {
-  a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.wait) &&
-                aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
+  a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.adm_scratch) &&
+                aligned16(a.wait) && aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
   if (policy & CONVGPU_DISPATCH_LITERAL) variant = CONVGPU_KERNEL_WARP_PER_TRACE;
   if (variant == CONVGPU_KERNEL_AUTO) {
     variant = auto_variant(a.count, policy);
@@ -141,7 +141,7 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   if (!out) return -EINVAL;
   if (out->range_digest && out->range_size == 0) return -EINVAL;
   if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT &&
-      (traces->n_containers != 64 || traces->n_ops != 4 || !out->admit_tick))
+      (traces->n_containers != 64 || traces->n_ops != 4 || (!out->admit_tick && !out->admit_scratch)))
     return -EINVAL;
   if (n == 0) return 0;  // no-op: array pointers may be NULL
   if ((rc = validate_arrays(traces))) return rc;
@@ -152,16 +152,17 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   if (!opt_device_ptr(out->admit_tick) || !opt_device_ptr(out->admit_rank) ||
       !opt_device_ptr(out->wait) || !opt_device_ptr(out->finish) ||
       !opt_device_ptr(out->summary) || !opt_device_ptr(out->stats) ||
-      !opt_device_ptr(out->range_digest))
+      !opt_device_ptr(out->range_digest) || !opt_device_ptr(out->admit_scratch))
     return -EINVAL;
   convgpu::ReplayArgs a = make_args(traces, n, capacity_mib);
   a.admit_tick = out->admit_tick; a.admit_rank = out->admit_rank;
   a.wait = out->wait; a.finish = out->finish;
   a.summary = out->summary; a.stats = out->stats;
   a.range_digest = out->range_digest; a.range_size = out->range_size;
+  a.adm_scratch = out->admit_scratch;
   if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT) {
-    a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.wait) &&
-                  aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
+    a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.adm_scratch) &&
+                  aligned16(a.wait) && aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
     if (!convgpu::lpt16_supported(a)) return -EINVAL;
   }
   cudaError_t e = launch_any(a, policy, traces->kernel_variant, (cudaStream_t)out->stream);
@@ -297,7 +298,7 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
-      a.admit_tick = adm_scratch;
+      a.adm_scratch = adm_scratch;  // admissions only; no per-container outputs
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
       e = launch_any(a, pols[q], ht->kernel_variant, cs);
     }
@@ -320,6 +321,15 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
   if (e == cudaSuccess) e = cudaEventRecord(back_done, back);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, back_done, 0);
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+  if (e != cudaSuccess) {
+    // an error mid-way: copies and kernels already enqueued may still read the
+    // caller's pinned buffers and write its workspace, which the caller frees
+    // or reuses once we return, so drain every stream before tearing down
+    // (secondary errors ignored; the first one is reported)
+    if (copy) cudaStreamSynchronize(copy);
+    if (back) cudaStreamSynchronize(back);
+    cudaStreamSynchronize(cs);
+  }
   for (int b = 0; b < 2; ++b) {
     if (h2d[b]) cudaEventDestroy(h2d[b]);
     if (kdone[b]) cudaEventDestroy(kdone[b]);

@@ -150,6 +150,16 @@ void handle_one(int idx, const convgpu_msg_t& m) {
     return;
   }
   const int c = k.container;
+  // a process that said EXIT (or whose container finished) owns no memory any
+  // more: an allocation or free from it would charge a finished container
+  // whose memory has gone back to the pool, so it is refused
+  if ((m.type == CONVGPU_MSG_ALLOC || m.type == CONVGPU_MSG_ALLOC_DONE ||
+       m.type == CONVGPU_MSG_ALLOC_FAIL || m.type == CONVGPU_MSG_FREE ||
+       m.type == CONVGPU_MSG_FREE_BYTES) &&
+      (k.exited || g_s->get((uint32_t)c).done)) {
+    send_reply(k, CONVGPU_ST_PROTOCOL, m.type);
+    return;
+  }
   switch (m.type) {
     case CONVGPU_MSG_HELLO: {
       if (k.container >= 0) { send_reply(k, CONVGPU_ST_PROTOCOL, m.type); return; }
@@ -302,10 +312,18 @@ int main(int argc, char** argv) {
         close(g_conns[i].fd);
         g_conns[i].fd = -1;
         if (g_conns[i].container >= 0) {
-          ContainerInfo& ci = g_ci[g_conns[i].container];
+          const int c = g_conns[i].container;
+          ContainerInfo& ci = g_ci[c];
+          const bool head = !ci.queue.empty() && ci.queue.front() == i;
           for (auto it = ci.queue.begin(); it != ci.queue.end(); ++it)
             if (*it == i) { ci.queue.erase(it); break; }
+          // its ALLOC paused the container: withdraw that request, so the
+          // next queued one goes through its own admission check (alloc())
+          // instead of inheriting the dead request's grant on resume
+          if (head) g_s->cancel_pause((uint32_t)c);
           process_exit(g_conns[i]);
+          if (!g_s->get((uint32_t)c).done) pump(c);
+          deliver_resumed();
         }
         continue;
       }

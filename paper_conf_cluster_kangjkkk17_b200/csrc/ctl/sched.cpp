@@ -99,6 +99,17 @@ void Scheduler::finish(uint32_t c) {
   dispatch();
 }
 
+bool Scheduler::cancel_pause(uint32_t c) {
+  Container& k = cs_[c];
+  if (!k.paused) return false;
+  k.paused = false;
+  k.pend = 0;
+  // a resume of c recorded in this step would now deliver a grant to the
+  // next queued request without its own admission check
+  resumed_.erase(std::remove(resumed_.begin(), resumed_.end(), c), resumed_.end());
+  return true;
+}
+
 int Scheduler::select() {
   int best = -1;
   for (uint32_t c = 0; c < cs_.size(); ++c) {

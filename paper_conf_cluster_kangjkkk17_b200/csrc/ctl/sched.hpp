@@ -45,6 +45,10 @@ class Scheduler {
   bool free_bytes(uint32_t c, uint64_t r);
   // FINISH (R18): release everything the container holds.
   void finish(uint32_t c);
+  // The process whose ALLOC paused container c went away before the reply:
+  // withdraw that request (c leaves the paused set; its assignment and, if it
+  // is the fill target, its target role stay).  Returns true if c was paused.
+  bool cancel_pause(uint32_t c);
   // Containers resumed by the last step, in resume order (their withheld
   // ALLOC replies are due).
   std::vector<uint32_t> take_resumed();

@@ -41,6 +41,14 @@ pthread_mutex_t g_mu = PTHREAD_MUTEX_INITIALIZER;  // one request in flight per 
 // A call made while this thread is already inside the shim (e.g. a runtime
 // call that reaches a driver entry point we also wrap) passes straight
 // through: it is part of the outer request, and g_mu is not recursive.
+//
+// Known limitation: g_mu is held across the blocking request, so while one
+// thread's cudaMalloc is paused (reply withheld) every other thread of
+// the process that calls into the shim (cudaFree, cudaMemGetInfo, the
+// teardown's __cudaUnregisterFatBinary) waits until the scheduler resumes it.
+// Replies carry no request id, so one connection cannot have two requests in
+// flight; a process exiting while a worker thread is paused therefore blocks
+// in teardown until resumed (or until the daemon drops the connection).
 __thread int t_depth = 0;
 struct Lock {
   const bool outer;
@@ -246,7 +254,15 @@ EXPORT void __cudaUnregisterFatBinary(void** handle) {
   {
     Lock lk;
     convgpu_reply_t r;
-    if (lk.outer && g_state == 1) rpc(CONVGPU_MSG_EXIT, 0, 0, &r);  // the process is ending
+    if (lk.outer && g_state == 1) {
+      rpc(CONVGPU_MSG_EXIT, 0, 0, &r);  // the process is ending
+      // the container's memory is being released: later calls (teardown
+      // allocations, another fat binary's unregistration) pass straight
+      // through instead of charging a finished container
+      g_state = -1;
+      close(g_fd);
+      g_fd = -1;
+    }
   }
   if (fn) fn(handle);
 }

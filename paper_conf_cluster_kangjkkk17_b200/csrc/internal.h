@@ -27,7 +27,11 @@ struct ReplayArgs {
   uint64_t grid_override;  // 0 = occupancy-sized persistent grid
   uint32_t per_sm_cap;     // tuning knob (env CONVGPU_PER_SM_CAP): at most this many CTAs per SM
   uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
-  uint32_t only_marked;    // lane kernel: replay only traces with admit_tick[i*n] == kLpt16Mark
+  uint32_t only_marked;    // lane kernel: replay only traces with adm_buf()[i*n] == kLpt16Mark
+  uint32_t* adm_scratch;   // compact kernel: admissions during the replay when admit_tick == NULL
+
+  // where the compact kernel keeps admissions (and its fallback marks)
+  __host__ __device__ uint32_t* adm_buf() const { return admit_tick ? admit_tick : adm_scratch; }
 };
 
 // admit_tick[i*n] of a trace the compact kernel left to the 32-bit lane kernel

@@ -373,7 +373,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
 #pragma unroll
       for (int u = 0; u < 8; ++u) {
         const uint64_t jj = j + (uint64_t)u * T;
-        m[u] = jj < p.count ? p.admit_tick[jj * n] : 0u;
+        m[u] = jj < p.count ? p.adm_buf()[jj * n] : 0u;
       }
 #pragma unroll
       for (int u = 0; u < 8; ++u)

@@ -8,8 +8,9 @@
 //    warp): key (u32), ust (u32: used 16 | op index 3 | FIRST | PAUSED |
 //    ADMITTED | op kinds 2 x K), sd (u32: size of the current op, saturated
 //    to 16 bits | delta of the next op 16), L (u16, [container][lane]);
-//  * no admission word: an admission is stored straight to admit_tick (as
-//    tick << 6 | rank) and read back by the epilogue; the finish tick lives
+//  * no admission word: an admission is stored straight to admit_tick, or to
+//    the caller's admission scratch when admit_tick is not requested (as
+//    tick << 6 | rank), and read back by the epilogue; the finish tick lives
 //    in the container's key after FINISH (0x80000000 | tick) and a paused
 //    container's key is 0xC0000000 (Recent-Fit: | the next container down the
 //    suspension stack, which is thereby a linked list needing no extra
@@ -28,7 +29,7 @@
 // ticks and its horizon (R19) < 2^25 (BASELINE configs [1]-[4] all do; the
 // 16-bit fields are then exact: a saturated size is above every limit, so it
 // is rejected / flagged exactly as the full size would be).  Other traces are
-// marked (admit_tick[trace][0] = kMark) and replayed by the 32-bit
+// marked (admissions[trace][0] = kMark) and replayed by the 32-bit
 // lane-per-trace kernel in a second launch that skips unmarked traces.
 // Semantics are identical to replay_lpt.cu / replay.cu; every
 // GPU parity test runs this kernel against the oracle too.
@@ -165,7 +166,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     const uint4* L4 = reinterpret_cast<const uint4*>(p.limit + ti * n);
     trace_delta = p.delta + ti * (uint64_t)K * n;
     trace_arg = p.arg + ti * (uint64_t)K * n;
-    adm_out = p.admit_tick + ti * n;
+    adm_out = p.adm_buf() + ti * n;
     const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
     const uint4* R4 = reinterpret_cast<const uint4*>(trace_arg);
     uint32_t bad = 0, lsum = 0, amax = 0, prev = 0, lmax = 0, dmax = 0;
@@ -209,7 +210,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     // not representable in the 16-bit fields: the 32-bit kernel replays it
     skip = bad == 0 && (lmax > 0xFFFEu || dmax > 0xFFFFu || amax + lsum >= kCompactHorizon);
-    if (skip) adm_out[0] = kLpt16Mark;
+    // container 0's slot doubles as the fallback mark; clear a stale mark a
+    // previous call may have left in caller scratch (admissions of container
+    // 0 are only read back when it was admitted, so 0 is harmless)
+    adm_out[0] = skip ? kLpt16Mark : 0u;
     if (POLICY == CONVGPU_BEST_FIT) {
       uint32_t v[64];
 #pragma unroll
@@ -274,7 +278,8 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       }
       // streaming stores (evict-first): outputs are not re-read, inputs of the
       // traces in flight should stay in L2
-      __stcs(reinterpret_cast<uint4*>(p.admit_tick + ob) + q, make_uint4(at[0], at[1], at[2], at[3]));
+      if (p.admit_tick)
+        __stcs(reinterpret_cast<uint4*>(p.admit_tick + ob) + q, make_uint4(at[0], at[1], at[2], at[3]));
       if (p.admit_rank)
         __stcs(reinterpret_cast<unsigned int*>(p.admit_rank + ob) + q,
                ar[0] | (ar[1] << 8) | (ar[2] << 16) | (ar[3] << 24));
@@ -604,7 +609,7 @@ static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
 }  // namespace lpt16
 
 bool lpt16_supported(const ReplayArgs& a) {
-  return a.n == lpt16::N && a.K == lpt16::KOPS && a.admit_tick != nullptr && a.aligned16;
+  return a.n == lpt16::N && a.K == lpt16::KOPS && a.adm_buf() != nullptr && a.aligned16;
 }
 
 cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream) {

@@ -114,3 +114,55 @@ def test_multi_process_container_and_disconnect():
         other.close()
         p1.close()
         cc.close()
+
+
+def test_disconnect_while_paused_withdraws_the_request():
+    """A process whose ALLOC paused its container disconnects while another
+    process of the same container has an ALLOC queued: the dead request is
+    withdrawn, and the queued one goes through its own admission check
+    instead of inheriting the dead request's grant (so the container never
+    uses more than its declared limit, P:7)."""
+    ctl, path, d = _daemon(100, ovh=0)
+    with d:
+        cc = ctl.Client(path, pid=0)
+        a = ctl.Client(path, pid=1)
+        assert a.call(ctl.HELLO, 60, 1)[2] == 0  # admitted with 60
+        b1, b2 = ctl.Client(path, pid=2), ctl.Client(path, pid=3)
+        assert b1.call(ctl.HELLO, 50, 2)[2] == 1  # 40 of 50: fill target
+        assert b2.call(ctl.HELLO, 50, 2)[2] == 1
+        b1.send(ctl.ALLOC, 45)  # 45 > 40 assigned: paused (P:139)
+        b2.send(ctl.ALLOC, 40)  # queued behind b1's request
+        cc.call(ctl.SYNC)
+        assert b2.recv(block=False) is None
+        b1.close()  # b1 dies with its request paused
+        rep = b2.recv()  # b2's own request: 40 <= 40 assigned, granted
+        assert rep[:2] == (ctl.OK, ctl.ALLOC)
+        assert cc.call(ctl.INFO, 1)[2:4] == (40, 40)
+        assert b2.call(ctl.ALLOC, 20)[0] == ctl.REJECT  # 60 > limit 50
+        assert cc.call(ctl.INFO, 1)[2:4] == (40, 40)
+        assert a.call(ctl.EXIT)[0] == ctl.OK  # A's 60 returns; B filled to 50
+        assert cc.call(ctl.INFO, 1)[2:5] == (50, 40, 1)
+        b2.close()
+        a.close()
+        assert cc.call(ctl.STATS)[2] == 100
+        cc.close()
+
+
+def test_alloc_after_exit_is_refused():
+    """After EXIT the process's container has given its memory back: a later
+    ALLOC / FREE from that connection is a protocol error and charges
+    nothing, so the pool is whole again after the disconnect."""
+    ctl, path, d = _daemon(100, ovh=0)
+    with d:
+        cc = ctl.Client(path, pid=0)
+        p = ctl.Client(path, pid=1)
+        assert p.call(ctl.HELLO, 60, 1)[0] == ctl.OK
+        assert cc.call(ctl.STATS)[2] == 40
+        assert p.call(ctl.EXIT)[0] == ctl.OK
+        assert cc.call(ctl.STATS)[2] == 100
+        assert p.call(ctl.ALLOC, 10)[0] == ctl.PROTOCOL
+        assert p.call(ctl.FREE_BYTES, 1)[0] == ctl.PROTOCOL
+        assert p.call(ctl.ALLOC_DONE, 0x10, 10)[0] == ctl.PROTOCOL
+        p.close()
+        assert cc.call(ctl.STATS)[2] == 100
+        cc.close()

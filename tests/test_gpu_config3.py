@@ -29,7 +29,11 @@ def _golden():
 
 
 @pytest.mark.parametrize("policy", ["fifo", "best_fit", "recent_fit", "random_fit"])
-def test_config3_range_digests(policy):
+@pytest.mark.parametrize("kernel", ["lane16", "lane"])
+def test_config3_range_digests(policy, kernel):
+    """kernel: "lane16" = the compact kernel bench.py times (summary-only
+    through the admission scratch, as AUTO picks it), "lane" = the 32-bit
+    lane kernel."""
     import torch
 
     import paper_conf_cluster_kangjkkk17_b200 as cg
@@ -54,8 +58,9 @@ def test_config3_range_digests(policy):
                        buf.op_arg[:hi - lo])
         cg.generate(w.gen, lo, hi - lo, out=tr)
         out = cg.alloc_out(hi - lo, w.gen.n, full=False, summary=False, range_count=nr,
-                           range_size=rs)
-        cg.replay(tr, w.cap, policy, out, rand_seed=w.rand_seed)
+                           range_size=rs, scratch=kernel == "lane16")
+        cg.replay(tr, w.cap, policy, out, rand_seed=w.rand_seed,
+                  kernel="auto" if kernel == "lane16" else kernel)
         torch.cuda.synchronize()
         rd = out.range_digest.cpu().numpy().view(np.uint64)
         st = cg.stats_dict(out.stats_np())

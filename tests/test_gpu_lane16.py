@@ -131,8 +131,9 @@ def test_lane16_rejects_unsupported_shapes(cg):
         cg.replay(tr, w.cap, "fifo", cg.alloc_out(64, 16), kernel="lane16")
     w2 = W.CONFIGS["c2"]
     tr = cg.generate(w2.gen, 0, 64)
-    with pytest.raises(cg.ConvgpuError):  # admit_tick is the admission scratch
-        cg.replay(tr, w2.cap, "fifo", cg.alloc_out(64, 64, full=False), kernel="lane16")
+    with pytest.raises(cg.ConvgpuError):  # neither admit_tick nor the admission scratch
+        cg.replay(tr, w2.cap, "fifo", cg.alloc_out(64, 64, full=False, scratch=False),
+                  kernel="lane16")
     with pytest.raises(cg.ConvgpuError):  # R1-LIT runs on the warp kernel only
         cg.replay(tr, w2.cap, "fifo+literal", cg.alloc_out(64, 64), kernel="lane16")
 
@@ -197,3 +198,54 @@ def test_lane16_fused_arrival_step(cg, orc, policy, cap, ovh):
     flags = ref["flags"]
     assert (flags & 8).any() and (flags == 0).sum() > 100
     assert int(ref["stats"]["n_select"]) > 0 and int(ref["stats"]["n_rejected"]) > 0
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_summary_only_with_scratch(cg, orc, policy):
+    """Summary / stats / digest-only launches (no per-container outputs) run on
+    the compact kernel through the caller's admission scratch (ABI 4): config
+    [2] traces, rho = 8 traces (all through the marked 32-bit fallback) and
+    edge-case traces, each against the oracle's summaries and statistics."""
+    cases = []
+    w = W.CONFIGS["c2"]
+    cases.append((w.cap, 0, w.rand_seed, 5_000_000_000, cg.generate(w.gen, 5_000_000_000, 3_001),
+                  orc.replay_range(w, policy, 5_000_000_000, 5_003_001)))
+    w8 = W.rho_sweep(8, rand_seed=9)
+    cases.append((w8.cap, 0, 9, 0, cg.generate(w8.gen, 0, 700), orc.replay_range(w8, policy, 0, 700)))
+    b = W.random_batch(77, 600, 64, 4, 300, ovh=5, mode="mixed", limit_choices=range(0, 301))
+    cases.append((300, 5, 4, 17, cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg,
+                                                       trace_id_base=17),
+                  orc.replay_batch(b, 300, policy, tid_base=17, rand_seed=4, ovh=5)))
+    for cap, ovh, seed, _, tr, ref in cases:
+        for kernel in ("lane16", "auto"):
+            out = _gpu_replay(cg, tr, cap, policy, seed=seed, ovh=ovh, full=False, kernel=kernel)
+            assert out.admit_scratch is not None and out.admit_tick is None
+            _compare(cg, out, ref, full=False)
+            _compare_stats(cg, out, ref["stats"])
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_scratch_reuse_clears_stale_marks(cg, orc, policy):
+    """A scratch buffer reused across calls: the first call leaves fallback
+    marks (rho = 8 limits exceed the 16-bit fields) in the slots that the
+    second call's statically flagged traces never write; those traces must
+    not be replayed a second time by the fallback pass."""
+    import torch
+    w8 = W.rho_sweep(8, rand_seed=1)
+    N = 512
+    tr8 = cg.generate(w8.gen, 0, N)
+    scratch = torch.empty(N, 64, dtype=torch.int32, device="cuda")
+    out = cg.alloc_out(N, 64, full=False, scratch=False)
+    out.admit_scratch = scratch
+    cg.replay(tr8, w8.cap, policy, out, rand_seed=1, kernel="lane16")
+    torch.cuda.synchronize()
+    assert (scratch[:, 0].cpu().numpy().view(np.uint32) == 0xFFFFFFFE).any()
+    b = W.random_batch(3, N, 64, 4, 200, mode="biglimit", limit_choices=range(0, 201))
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
+    ref = orc.replay_batch(b, 200, policy)
+    out2 = cg.alloc_out(N, 64, full=False, scratch=False)
+    out2.admit_scratch = scratch
+    cg.replay(tr, 200, policy, out2, kernel="lane16")
+    torch.cuda.synchronize()
+    _compare(cg, out2, ref, full=False)
+    _compare_stats(cg, out2, ref["stats"])

@@ -26,10 +26,10 @@ KERNELS = ["warp", "lane"]
 
 
 def _gpu_replay(cg, tr, cap, policy, seed=0, ovh=0, full=True, range_size=0, range_count=0,
-                kernel="auto"):
+                kernel="auto", scratch=None):
     import torch
     out = cg.alloc_out(tr.count, tr.n, full=full, range_count=range_count,
-                       range_size=range_size)
+                       range_size=range_size, scratch=scratch)
     cg.replay(tr, cap, policy, out, rand_seed=seed, ovh=ovh, kernel=kernel)
     torch.cuda.synchronize()
     return out
