@@ -209,7 +209,7 @@ def test_lane16_summary_only_with_scratch(cg, orc, policy):
     cases = []
     w = W.CONFIGS["c2"]
     cases.append((w.cap, 0, w.rand_seed, 5_000_000_000, cg.generate(w.gen, 5_000_000_000, 3_001),
-                  orc.replay_range(w, policy, 5_000_000_000, 5_003_001)))
+                  orc.replay_range(w, policy, 5_000_000_000, 5_000_003_001)))
     w8 = W.rho_sweep(8, rand_seed=9)
     cases.append((w8.cap, 0, 9, 0, cg.generate(w8.gen, 0, 700), orc.replay_range(w8, policy, 0, 700)))
     b = W.random_batch(77, 600, 64, 4, 300, ovh=5, mode="mixed", limit_choices=range(0, 301))
