@@ -53,3 +53,30 @@ def test_two_rank_config3_prefix_checked_against_oracle():
     par = d["parity"]
     assert par["equal"] is True and par["ranges"] == 16, par
     assert d["config"]["traces_total"] == 4 << 20 and d["config"]["traces_per_gpu"] == 2 << 20
+
+
+def test_rho_sweep_two_ranks_equals_one(tmp_path):
+    """Config [4] sharded over ranks: the statistics all-reduced over two
+    ranks (each replaying half of every point's trace ids) equal one rank
+    replaying all of them, run by run (digest sums, events, flags)."""
+    one, two = tmp_path / "one.json", tmp_path / "two.json"
+    common = ["--traces", "20000", "--seeds", "2", "--lit-seeds", "1", "--rhos", "2,8"]
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "scripts", "rho_sweep.py")] + common +
+                       ["--out", str(one)], capture_output=True, text=True, timeout=900, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    env = dict(os.environ, CONVGPU_DIST_BACKEND="gloo", OMP_NUM_THREADS="1")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+                        "--nproc-per-node", "2", "--master-addr", "127.0.0.1", "--master-port",
+                        "29533", os.path.join(ROOT, "scripts", "rho_sweep.py")] + common +
+                       ["--out", str(two)], capture_output=True, text=True, timeout=900, cwd=ROOT,
+                       env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    a, b = json.loads(one.read_text()), json.loads(two.read_text())
+    assert b["n_gpus"] == 2
+    for part in ("runs",):
+        for x, y in zip(a[part], b[part]):
+            assert (x["rho"], x["policy"], x["seed"]) == (y["rho"], y["policy"], y["seed"])
+            assert x["digest_sum"] == y["digest_sum"] and x["events"] == y["events"]
+            assert x["flag_count"] == y["flag_count"]
+    for x, y in zip(a["literal"]["runs"], b["literal"]["runs"]):
+        assert x["digest_sum"] == y["digest_sum"] and x["deadlock_share"] == y["deadlock_share"]
