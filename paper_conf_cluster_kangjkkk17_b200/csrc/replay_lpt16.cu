@@ -39,14 +39,11 @@
 #include "common.cuh"
 #include "internal.h"
 #include "lpt_util.cuh"
-#include "oem64.cuh"
 
 namespace convgpu {
 namespace lpt16 {
 
 using lpt::ffs64;
-using lpt::fls64;
-using lpt::lowmask64;
 using lpt::shl_c;
 using lpt::sts_if;
 
@@ -68,17 +65,23 @@ constexpr uint32_t kNoC = 64u;
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kCompactHorizon = 1u << 25;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
+constexpr uint32_t kTmemCols = 128;
+ // 64 per warp, warps w and w + 4 share a lane quarter
 
 // bytes per lane (= per trace) and warps per CTA (one CTA per SM)
 __host__ __device__ constexpr uint32_t extra_bytes(int policy) {
-  return policy == CONVGPU_BEST_FIT ? N * 2u : 0u;  // Best-Fit: rank_of / pi bytes
+  return 0u;  // every policy's extra state lives in registers (Best-Fit: limit classes)
 }
 __host__ __device__ constexpr uint32_t lane_bytes(int policy) {
   return N * 14u + extra_bytes(policy) + 8u;  // + 2-word fetch staging slot
 }
 __host__ __device__ constexpr int warps_per_cta(int policy) {
-  return policy == CONVGPU_BEST_FIT ? 7 : 8;
+  return 8;
 }
+// Best-Fit keeps the trace's distinct declared limits ("classes") in
+// registers; a trace with more distinct limits than this is left to the
+// 32-bit kernel (marked), like one whose values exceed the 16-bit fields.
+constexpr int kBfClasses = 8;
 
 __device__ __forceinline__ uint32_t comp(const uint4& v, int j) {
   return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
@@ -106,16 +109,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // limits: u16 of container c of this lane at [c * 32 + lane] (one IMAD per
   // address; at most 2-way bank conflicts, between lanes 2j and 2j + 1)
   uint16_t* const s_L = reinterpret_cast<uint16_t*>(W0 + 3 * n * 32) + lane;
-  // Best-Fit: rank of container c in (L, index) order and container of rank
-  // r, bytes (byte e of this lane at [(e >> 2) * 128 + (e & 3)])
-  uint8_t* const s_rof = reinterpret_cast<uint8_t*>(W0 + (3 * n + n / 2) * 32) + lane * 4;
-  uint8_t* const s_pi = reinterpret_cast<uint8_t*>(W0 + (3 * n + n / 2 + n / 4) * 32) + lane * 4;
   // staging slot of the one-op-ahead fetch: {op word, delta of the op after}
   uint32_t* const s_stg = W0 + (3 * n + n / 2 + extra_bytes(POLICY) / 4) * 32 + lane;
 #define AT(arr, c) (arr)[(c) * 32u]
 #define LIM(c) s_L[(c) * 32u]
-#define ROF(c) s_rof[((c) >> 2) * 128u + ((c) & 3u)]
-#define PI(r) s_pi[((r) >> 2) * 128u + ((r) & 3u)]
 
   // A warp replays 32 consecutive traces per round; round-robin warp slots
   // run SM-first (slot = wib * gridDim + block), so the last, partial round
@@ -129,15 +126,42 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   unsigned long long racc_r = ~0ull, racc = 0;
 
   uint32_t gmin[8];
-  // arrival + sum of deltas per container, in registers (R17's wait = finish -
-  // base is then computed without re-reading the trace in the epilogue)
+  // arrival + sum of deltas per container (R17's wait = finish - base is then
+  // computed without re-reading the trace in the epilogue).  Computed in
+  // registers by init, parked in this thread's TMEM lane for the whole event
+  // loop (64 columns), read back for the epilogue: the loop does not carry 64
+  // registers for it.
   uint32_t base[64];
+  __shared__ uint32_t s_tmem;
+  if (wib == 0) lpt::tmem_alloc(&s_tmem, kTmemCols);
+  lpt::tmem_fence_before_sync();
+  __syncthreads();
+  lpt::tmem_fence_after_sync();
+  const uint32_t t_base = s_tmem + ((32u * (wib & 3u)) << 16) + (wib >> 2) * 64u;
+  auto park_base = [&]() {  // whole warp, converged
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < 4; ++q) lpt::tmem_st16(t_base + 16u * q, base + 16 * q);
+  };
+  auto fetch_base = [&]() {  // whole warp, converged
+    __syncwarp();
+    lpt::tmem_wait_st();
+#pragma unroll
+    for (int q = 0; q < 4; ++q) lpt::tmem_ld16(t_base + 16u * q, base + 16 * q);
+    lpt::tmem_wait_ld();
+  };
   uint32_t arr0 = 0;
-  uint32_t piv[8];
+  // Best-Fit (R3, R4): the trace's distinct limits in ascending order (unused
+  // slots 0xFFFFFFFF, above every free amount) and, per class, the mask of
+  // containers declaring that limit.  A paused non-target container has no
+  // memory assigned (R1: only the fill target is ever partial), so its
+  // shortfall is its limit: the Best-Fit choice is the lowest-index paused
+  // member of the highest class whose limit fits the free memory, else of
+  // the lowest class with a paused member.
+  uint32_t bl[kBfClasses], bm_lo[kBfClasses], bm_hi[kBfClasses];
   uint32_t free_mem = 0, target = kNoC, a_tg = 0, used_total = 0, rank = 0, draws = 0,
            n_rej = 0, n_sel = 0, peak_res = 0, peak_used = 0, flags = 0, live = 0, events = 0;
-  uint32_t pm_lo = 0, pm_hi = 0, pr_lo = 0, pr_hi = 0;
-  uint32_t eq_lo = 0, eq_hi = 0;  // Best-Fit: rank r has the same limit as rank r - 1
+  uint32_t pm_lo = 0, pm_hi = 0;
   uint32_t ru_head = kNoC;        // Recent-Fit: top of the suspension stack (linked
                                   // through the paused containers' keys)
   // the op fetched in the previous iteration: container, op word, delta
@@ -215,31 +239,56 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     // 0 are only read back when it was admitted, so 0 is harmless)
     adm_out[0] = skip ? kLpt16Mark : 0u;
     if (POLICY == CONVGPU_BEST_FIT) {
-      uint32_t v[64];
+      // distinct limits (unsorted while collected), with member masks
+      uint32_t ncls = 0;
 #pragma unroll
-      for (int c = 0; c < 64; ++c) v[c] = ((uint32_t)LIM(c) << 6) | (uint32_t)c;
-      // Batcher's odd-even merge sort network (oem64.cuh): 543
-      // compare-exchanges for 64 keys, literal indices, v stays in registers
-#define OEM_CE(a, b) { const uint32_t x = v[a], y = v[b]; v[a] = min(x, y); v[b] = max(x, y); }
-      OEM64_NETWORK(OEM_CE)
-#undef OEM_CE
+      for (int j = 0; j < kBfClasses; ++j) { bl[j] = 0xFFFFFFFFu; bm_lo[j] = 0; bm_hi[j] = 0; }
 #pragma unroll
-      for (int j = 0; j < 8; ++j) piv[j] = v[8 * j + 7] >> 6;
-      uint32_t prevL = 0xFFFFFFFFu;
-      eq_lo = eq_hi = 0;
+      for (int c = 0; c < 64; ++c) {
+        const uint32_t Lc = LIM(c), bit = 1u << (c & 31);
+        bool hit = false;
 #pragma unroll
-      for (int r = 0; r < 64; ++r) {
-        const uint32_t c = v[r] & 63u, Lc = v[r] >> 6;
-        if (Lc == prevL) { if (r < 32) eq_lo |= 1u << r; else eq_hi |= 1u << (r - 32); }
-        prevL = Lc;
-        ROF(c) = (uint8_t)r;
-        PI(r) = (uint8_t)c;
+        for (int j = 0; j < kBfClasses; ++j) {
+          const bool e = bl[j] == Lc;
+          hit |= e;
+          if (c < 32) bm_lo[j] |= e ? bit : 0u; else bm_hi[j] |= e ? bit : 0u;
+        }
+        if (!hit) {  // a new class (at most kBfClasses + 1 times per trace)
+#pragma unroll
+          for (int j = 0; j < kBfClasses; ++j) {
+            const bool e = (uint32_t)j == ncls;
+            bl[j] = e ? Lc : bl[j];
+            if (c < 32) bm_lo[j] |= e ? bit : 0u; else bm_hi[j] |= e ? bit : 0u;
+          }
+          ++ncls;
+        }
+      }
+      // sort the classes by limit (Batcher's network for 8 keys, 19 exchanges)
+#define BF_CE(a, b)                                                              \
+  {                                                                              \
+    const bool sw = bl[a] > bl[b];                                               \
+    const uint32_t x = bl[a], y = bm_lo[a], z = bm_hi[a];                        \
+    bl[a] = sw ? bl[b] : x; bm_lo[a] = sw ? bm_lo[b] : y; bm_hi[a] = sw ? bm_hi[b] : z; \
+    bl[b] = sw ? x : bl[b]; bm_lo[b] = sw ? y : bm_lo[b]; bm_hi[b] = sw ? z : bm_hi[b]; \
+  }
+      BF_CE(0, 1) BF_CE(2, 3) BF_CE(4, 5) BF_CE(6, 7)
+      BF_CE(0, 2) BF_CE(1, 3) BF_CE(4, 6) BF_CE(5, 7)
+      BF_CE(1, 2) BF_CE(5, 6) BF_CE(0, 4) BF_CE(3, 7)
+      BF_CE(1, 5) BF_CE(2, 6)
+      BF_CE(1, 4) BF_CE(3, 6)
+      BF_CE(2, 4) BF_CE(3, 5)
+      BF_CE(3, 4)
+#undef BF_CE
+      // more distinct limits than classes: the 32-bit kernel replays it
+      if (bad == 0 && ncls > (uint32_t)kBfClasses && !skip) {
+        skip = true;
+        adm_out[0] = kLpt16Mark;
       }
     }
     flags = bad;
     free_mem = cap; target = kNoC; a_tg = 0; used_total = 0; rank = 0; draws = 0;
     n_rej = 0; n_sel = 0; peak_res = 0; peak_used = 0; live = n; events = 0;
-    pm_lo = pm_hi = pr_lo = pr_hi = 0;
+    pm_lo = pm_hi = 0;
     pre_c = kNoC;
     ru_head = kNoC;
   };
@@ -325,6 +374,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
   if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
+  park_base();
   while (__any_sync(kFull, have)) {
     do {
       if (have && !tdone) {
@@ -398,11 +448,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const uint32_t pmask = pause ? 0xFFFFFFFFu : 0u;
             pm_lo |= shl_c(1u, c) & pmask;
             pm_hi |= shl_c(1u, c - 32u) & pmask;
-            if (POLICY == CONVGPU_BEST_FIT) {
-              const uint32_t rc = ROF(c);
-              pr_lo |= shl_c(1u, rc) & pmask;
-              pr_hi |= shl_c(1u, rc - 32u) & pmask;
-            }
             // Recent-Fit: push c on the suspension stack (its key links the old
             // top) unless it is the fill target, which resumes without a
             // selection (R1) and so must never be popped
@@ -437,27 +482,26 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             n_sel += ns ? 1u : 0u;
           } else if (target == kNoC) {
             uint32_t sel;
-            if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4
-              uint32_t gc = 0;
+            if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4 (classes: see bl above)
+              // ascending classes: the last fitting class with a paused
+              // member wins; descending: the last class with one is the lowest
+              uint32_t fl = 0, fh = 0, ml = 0, mh = 0;
 #pragma unroll
-              for (int j = 0; j < 8; ++j) gc += (piv[j] <= free_mem) ? 1u : 0u;
-              const uint32_t rb = min(gc, 7u) * 8u;
-              uint32_t in = 0;
+              for (int j = 0; j < kBfClasses; ++j) {
+                const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
+                const bool on = ((a | b) != 0u) && bl[j] <= free_mem;
+                fl = on ? a : fl;
+                fh = on ? b : fh;
+              }
 #pragma unroll
-              for (uint32_t j = 0; j < 8; ++j) in += ((uint32_t)LIM(PI(rb + j)) <= free_mem) ? 1u : 0u;
-              const uint32_t lo = (gc == 8u) ? 64u : rb + in;
-              uint32_t ml, mh;
-              lowmask64(lo, ml, mh);
-              const uint32_t fl = pr_lo & ml, fh = pr_hi & mh;
-              const uint32_t h = min(fls64(fl, fh), n - 1u);
-              // first rank of h's limit group: the highest rank <= h that
-              // starts a group (rank 0 always does)
-              uint32_t hl, hh, gl, gh;
-              lowmask64(h + 1u, hl, hh);
-              lowmask64(fls64(~eq_lo & hl, ~eq_hi & hh), gl, gh);
-              const uint32_t r_fit = ffs64(pr_lo & ~gl, pr_hi & ~gh);
-              const uint32_t r_min = ffs64(pr_lo, pr_hi);
-              sel = PI((fl | fh) ? r_fit : r_min);
+              for (int j = kBfClasses - 1; j >= 0; --j) {
+                const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
+                const bool on = (a | b) != 0u;
+                ml = on ? a : ml;
+                mh = on ? b : mh;
+              }
+              const bool fit = (fl | fh) != 0u;
+              sel = ffs64(fit ? fl : ml, fit ? fh : mh);
             } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
               // pop the suspension stack: paused containers leave the paused
               // set only by resuming, and only the target resumes, so popping
@@ -501,11 +545,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;
             pm_lo &= ~(shl_c(1u, tg) & rmask);
             pm_hi &= ~(shl_c(1u, tg - 32u) & rmask);
-            if (POLICY == CONVGPU_BEST_FIT) {
-              const uint32_t rt = ROF(tg);
-              pr_lo &= ~(shl_c(1u, rt) & rmask);
-              pr_hi &= ~(shl_c(1u, rt - 32u) & rmask);
-            }
             stg_if(adm_out + tg, (t << 6) | rank, full);
             rank += full ? 1u : 0u;
             target = full ? kNoC : target;
@@ -535,15 +574,15 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         }
       }
     } while (!__all_sync(kFull, !have || tdone));
+    fetch_base();
     if (have) {
       if (!skip) epilogue(i);
       i += T;
       have = i < p.count;
       if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
     }
+    park_base();
   }
-#undef PI
-#undef ROF
 #undef LIM
 #undef AT
 
@@ -576,6 +615,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       atomicMax(&Sg->max_peak_reserved, st_maxpk);
     }
   }
+  lpt::tmem_fence_before_sync();
+  __syncthreads();
+  lpt::tmem_fence_after_sync();
+  if (wib == 0) lpt::tmem_dealloc(s_tmem, kTmemCols);
 }
 
 template <int POLICY>

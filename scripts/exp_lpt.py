@@ -51,7 +51,9 @@ def main():
                 torch.cuda.synchronize()
                 best = min(best, e0.elapsed_time(e1))
             ms[pol] = round(best, 2)
-        print(f"{a.env}={v} {a.kernel} {tot_ev / (sum(ms.values()) / 1e3):.3e} ev/s {ms}", flush=True)
+        dig = ",".join("%04x" % (ref[p]["digest_sum"] >> 48) for p in W.POLICIES)
+        print(f"{a.env}={v} {a.kernel} {tot_ev / (sum(ms.values()) / 1e3):.3e} ev/s {ms} dig={dig}",
+              flush=True)
 
 
 if __name__ == "__main__":

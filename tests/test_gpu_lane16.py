@@ -249,3 +249,37 @@ def test_lane16_scratch_reuse_clears_stale_marks(cg, orc, policy):
     torch.cuda.synchronize()
     _compare(cg, out2, ref, full=False)
     _compare_stats(cg, out2, ref["stats"])
+
+
+CLASS_EDGE = [  # (cap, ovh, mode, count, distinct limits)
+    (256, 0, "valid", 700, 8),
+    (300, 5, "mixed", 700, 6),
+    (200, 1, "delayed", 500, 3),
+    (128, 0, "over", 500, 8),
+    (256, 0, "badfree", 400, 7),
+    (256, 0, "valid", 400, 9),   # one class too many: every trace goes to the fallback
+    (256, 2, "valid", 400, 1),   # all limits equal: Best-Fit = FIFO
+]
+
+
+@pytest.mark.parametrize("case", CLASS_EDGE, ids=lambda c: f"{c[2]}{c[0]}o{c[1]}k{c[4]}")
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_few_distinct_limits(cg, orc, policy, case):
+    """Edge-case programs over a handful of distinct limits, so that Best-Fit
+    traces stay on the compact kernel (its limit classes hold <= 8 distinct
+    limits; 9 sends the trace to the 32-bit fallback), element by element
+    against the oracle.  Limits include 0 and the capacity."""
+    cap, ovh, mode, count, k = case
+    rng = np.random.default_rng(31 * cap + k)
+    menu = ([0] + sorted(int(x) for x in rng.choice(np.arange(1, cap), size=k - 2, replace=False))
+            + [cap]) if k >= 2 else [cap // 2]
+    b = W.random_batch(5150 + cap + k, count, 64, 4, cap, ovh=ovh, mode=mode,
+                       limit_choices=menu)
+    base = 3_000_000_000 + cap * k
+    ref = orc.replay_batch(b, cap, policy, tid_base=base, rand_seed=9 + k, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=base)
+    out = _gpu_replay(cg, tr, cap, policy, seed=9 + k, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    if mode in ("valid", "delayed", "over"):
+        assert int(ref["stats"]["n_select"]) > 0
