@@ -235,6 +235,57 @@ int convgpu_replay_host(const convgpu_traces_t *host_traces, uint64_t n,
                         void *device_workspace, size_t workspace_bytes,
                         uint64_t chunk_traces, void *stream);
 
+/* ---- Compact 16-bit trace format (host end-to-end path) -------------------
+ * The same traces as convgpu_traces_t with every field in 16 bits and the op
+ * kinds in one byte per container: 21 B per container at n_ops = 4 instead of
+ * 40.  convgpu_replay_host is bound by the host-to-device copy of the traces
+ * (PCIe), not by the replay; convgpu_replay_host16 copies this format and
+ * restores the 32-bit layout on the device (an unpack kernel next to the
+ * replay), so the same replay reads about half the PCIe bytes.  Layout, trace
+ * i, container c, op k (n_ops <= 4):
+ *   arrival[i*n_containers + c], limit[i*n_containers + c]     u16
+ *   op_size[(i*n_ops + k)*n_containers + c]                    u16 (op_arg & 0x3FFFFFFF)
+ *   op_delta[(i*n_ops + k)*n_containers + c]                   u16
+ *   op_kinds[i*n_containers + c]                               u8: kind of op k in bits 2k, 2k+1
+ * A trace is representable when every arrival, limit, op size and delta is
+ * <= 0xFFFF (all BASELINE configs [0]-[4] are); convgpu_pack16 counts the
+ * values that are not. */
+typedef struct {
+  const uint16_t *arrival, *limit, *op_size, *op_delta; /* host (pinned for full speed) */
+  const uint8_t *op_kinds;
+  uint32_t n_containers;     /* 1..64 */
+  uint32_t n_ops;            /* 1..4 */
+  uint64_t trace_id_base, rand_seed;
+  uint32_t ctx_overhead_mib, kernel_variant; /* as in convgpu_traces_t */
+} convgpu_traces16_t;
+
+/* Writable DEVICE buffers of the 16-bit format. */
+typedef struct {
+  uint16_t *arrival, *limit, *op_size, *op_delta;
+  uint8_t *op_kinds;
+} convgpu_trace16_buffers_t;
+
+/* Pack n traces (DEVICE, 32-bit layout; the arrays of `src` are read, its other
+ * fields are ignored except n_containers / n_ops) into the 16-bit format in
+ * DEVICE buffers `dst`.  out_of_range (DEVICE u64, caller-zeroed, accumulated;
+ * NULL allowed) counts the values above 0xFFFF, whose packed copies are
+ * truncated: a batch is exact in the 16-bit format iff it stays 0.
+ * Asynchronous on `stream`.  Errors: -EINVAL (NULL, n_ops > 4, n_containers out
+ * of range, host pointers), -ENODEV, -EIO. */
+int convgpu_pack16(const convgpu_traces_t *src, uint64_t n, const convgpu_trace16_buffers_t *dst,
+                   uint64_t *out_of_range, void *stream);
+
+/* convgpu_replay_host for 16-bit HOST traces: the same chunked copy-in /
+ * replay-every-policy / summaries-back pipeline, plus one unpack kernel per
+ * chunk.  Same outputs, conventions and errors (n_ops > 4 is -EINVAL). */
+size_t convgpu_replay_host16_workspace(uint32_t n_containers, uint32_t n_ops,
+                                       uint64_t chunk_traces, uint32_t n_policies);
+int convgpu_replay_host16(const convgpu_traces16_t *host_traces, uint64_t n,
+                          uint32_t capacity_mib, uint32_t policy_mask,
+                          convgpu_summary_t *host_summary, convgpu_stats_t *host_stats,
+                          void *device_workspace, size_t workspace_bytes,
+                          uint64_t chunk_traces, void *stream);
+
 /* ---- NEXT-3: the wrapper module's size semantics ----------
  * PAPER.md §III-C: the wrapper intercepts the allocation APIs of Table II
  * and "calculates adjusted allocate size before checking

@@ -74,9 +74,23 @@ class BuffersT(C.Structure):
                 ("op_arg", C.c_void_p)]
 
 
+class Traces16T(C.Structure):
+    _fields_ = [("arrival", C.c_void_p), ("limit", C.c_void_p), ("op_size", C.c_void_p),
+                ("op_delta", C.c_void_p), ("op_kinds", C.c_void_p),
+                ("n_containers", C.c_uint32), ("n_ops", C.c_uint32),
+                ("trace_id_base", C.c_uint64), ("rand_seed", C.c_uint64),
+                ("ctx_overhead_mib", C.c_uint32), ("kernel_variant", C.c_uint32)]
+
+
+class Buffers16T(C.Structure):
+    _fields_ = [("arrival", C.c_void_p), ("limit", C.c_void_p), ("op_size", C.c_void_p),
+                ("op_delta", C.c_void_p), ("op_kinds", C.c_void_p)]
+
+
 EXPORTS = ("convgpu_replay", "convgpu_generate", "convgpu_replay_host",
            "convgpu_replay_host_workspace", "convgpu_wrap_ops", "convgpu_launches_per_call",
-           "convgpu_strerror", "convgpu_abi_version")
+           "convgpu_strerror", "convgpu_abi_version", "convgpu_pack16", "convgpu_replay_host16",
+           "convgpu_replay_host16_workspace")
 
 # NEXT-3 API records (include/convgpu.h convgpu_api_t / convgpu_api_op_t)
 API = {"malloc": 0, "malloc_managed": 1, "malloc_pitch": 2, "malloc_3d": 3, "free": 4,
@@ -106,6 +120,14 @@ def lib():
         L.convgpu_replay_host_workspace.restype = C.c_size_t
         L.convgpu_wrap_ops.argtypes = [C.c_void_p, C.c_uint64, C.c_uint32, C.c_uint32, C.c_uint32,
                                        C.c_void_p, C.c_void_p]
+        L.convgpu_pack16.argtypes = [C.POINTER(TracesT), C.c_uint64, C.POINTER(Buffers16T),
+                                     C.c_void_p, C.c_void_p]
+        L.convgpu_replay_host16.argtypes = [C.POINTER(Traces16T), C.c_uint64, C.c_uint32,
+                                            C.c_uint32, C.c_void_p, C.c_void_p, C.c_void_p,
+                                            C.c_size_t, C.c_uint64, C.c_void_p]
+        L.convgpu_replay_host16_workspace.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64,
+                                                      C.c_uint32]
+        L.convgpu_replay_host16_workspace.restype = C.c_size_t
         L.convgpu_strerror.argtypes = [C.c_int]
         L.convgpu_strerror.restype = C.c_char_p
         _lib = L
@@ -337,8 +359,97 @@ def replay_host(arrival, limit, delta, arg, capacity: int, policies=("fifo",), *
     return stats
 
 
-def host_workspace_bytes(n: int, K: int, chunk: int, n_policies: int = 1) -> int:
-    return int(lib().convgpu_replay_host_workspace(n, K, chunk, n_policies))
+def host_workspace_bytes(n: int, K: int, chunk: int, n_policies: int = 1, packed: bool = False) -> int:
+    f = lib().convgpu_replay_host16_workspace if packed else lib().convgpu_replay_host_workspace
+    return int(f(n, K, chunk, n_policies))
+
+
+# ---------------------------------------------------------------- 16-bit format
+@dataclass
+class Traces16:
+    """Traces in the compact 16-bit format of include/convgpu.h
+    (convgpu_traces16_t): int16 views of u16 arrival / limit [N, n], op_size /
+    op_delta [N, K, n]; uint8 op_kinds [N, n].  Device or (pinned) host."""
+    arrival: "torch.Tensor"
+    limit: "torch.Tensor"
+    op_size: "torch.Tensor"
+    op_delta: "torch.Tensor"
+    op_kinds: "torch.Tensor"
+
+    @property
+    def count(self) -> int:
+        return self.arrival.shape[0]
+
+    @property
+    def n(self) -> int:
+        return self.arrival.shape[1]
+
+    @property
+    def K(self) -> int:
+        return self.op_size.shape[1]
+
+    def nbytes(self) -> int:
+        return sum(t.numel() * t.element_size() for t in
+                   (self.arrival, self.limit, self.op_size, self.op_delta, self.op_kinds))
+
+    def pin(self) -> "Traces16":
+        """A pinned host copy (the e2e input)."""
+        import torch
+        cp = lambda t: torch.empty(t.shape, dtype=t.dtype, pin_memory=True).copy_(t)  # noqa: E731
+        return Traces16(*(cp(t) for t in (self.arrival, self.limit, self.op_size, self.op_delta,
+                                          self.op_kinds)))
+
+
+def pack16(traces: Traces, stream=None) -> tuple:
+    """Pack device traces into the 16-bit format on the device
+    (convgpu_pack16).  Returns (Traces16, out_of_range tensor): the packed
+    batch is exact iff out_of_range (int64[1], read after synchronising) is 0."""
+    import torch
+    N, n, K = traces.count, traces.n, traces.K
+    dev = traces.arrival.device
+    e = lambda *sh: torch.empty(*sh, dtype=torch.int16, device=dev)  # noqa: E731
+    t16 = Traces16(e(N, n), e(N, n), e(N, K, n), e(N, K, n),
+                   torch.empty(N, n, dtype=torch.uint8, device=dev))
+    oor = torch.zeros(1, dtype=torch.int64, device=dev)
+    buf = Buffers16T(t16.arrival.data_ptr(), t16.limit.data_ptr(), t16.op_size.data_ptr(),
+                     t16.op_delta.data_ptr(), t16.op_kinds.data_ptr())
+    _check(lib().convgpu_pack16(C.byref(traces.struct()), N, C.byref(buf), oor.data_ptr(),
+                                _stream_handle(stream)), "convgpu_pack16")
+    return t16, oor
+
+
+def replay_host16(t16: Traces16, capacity: int, policies=("fifo",), *, trace_id_base=0,
+                  rand_seed=0, ovh=0, chunk: int = 1 << 15, summary: Optional[np.ndarray] = None,
+                  workspace=None, stream=None, kernel: str = "auto"):
+    """End-to-end replay of HOST traces in the 16-bit format
+    (convgpu_replay_host16); as replay_host otherwise."""
+    import torch
+    for t in (t16.arrival, t16.limit, t16.op_size, t16.op_delta, t16.op_kinds):
+        if t.is_cuda or not t.is_contiguous():
+            raise ConvgpuError("replay_host16 expects contiguous host tensors")
+    if isinstance(policies, (str, int)):
+        policies = (policies,)
+    mask = 0
+    for q in policies:
+        mask |= 1 << _pol(q)
+    npol = bin(mask).count("1")
+    N, n, K = t16.count, t16.n, t16.K
+    tr = Traces16T(t16.arrival.data_ptr(), t16.limit.data_ptr(), t16.op_size.data_ptr(),
+                   t16.op_delta.data_ptr(), t16.op_kinds.data_ptr(), n, K, trace_id_base,
+                   rand_seed, ovh, KERNEL[kernel])
+    need = host_workspace_bytes(n, K, chunk, npol, packed=True)
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device="cuda")
+    stats = np.zeros(npol, STATS_DTYPE)
+    sp = None
+    if summary is not None:
+        assert summary.dtype == SUMMARY_DTYPE and summary.shape == (npol, N)
+        assert summary.flags["C_CONTIGUOUS"]
+        sp = summary.ctypes.data
+    _check(lib().convgpu_replay_host16(C.byref(tr), N, capacity, mask, sp, stats.ctypes.data,
+                                       workspace.data_ptr(), workspace.numel(), chunk,
+                                       _stream_handle(stream)), "convgpu_replay_host16")
+    return stats
 
 
 def stats_dict(rec) -> dict:

@@ -10,7 +10,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 SO = os.path.join(PKG, "libconvgpu.so")
-SOURCES = ["replay.cu", "replay_lpt.cu", "replay_lpt16.cu", "generate.cu", "wrap.cu", "abi.cu"]
+SOURCES = ["replay.cu", "replay_lpt.cu", "replay_lpt16.cu", "generate.cu", "wrap.cu", "pack16.cu",
+           "abi.cu"]
 HEADERS = ["common.cuh", "internal.h", "lpt_util.cuh", "oem64.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",

@@ -202,46 +202,94 @@ int convgpu_wrap_ops(const convgpu_api_op_t* api, uint64_t n, uint32_t n_contain
 }
 
 // ---------------------------------------------------------------- host e2e
-// Workspace layout (256-B aligned pieces): 2 x {arrival, limit, delta, arg}
-// chunk buffers, 2 x n_policies summary chunks, n_policies stats structs, one
-// chunk of per-container admission scratch.
+// Workspace layout (256-B aligned pieces).  32-bit format: 2 x {arrival,
+// limit, delta, arg} chunk buffers (double-buffered copy-in).  16-bit format:
+// 2 x {arrival16, limit16, size16, delta16, kinds8} copy-in buffers and one
+// 32-bit chunk set the unpack kernel writes (the replays of chunk j and the
+// unpack of chunk j + 1 are ordered on the caller's stream).  Then 2 x
+// n_policies summary chunks, n_policies stats structs and one chunk of
+// per-container admission scratch.
 static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
-size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops, uint64_t chunk,
-                                     uint32_t n_policies) {
-  const size_t cn = align256(chunk * n_containers * 4);
-  const size_t ckn = align256(chunk * n_containers * n_ops * 4);
-  return 2 * (2 * cn + 2 * ckn) + 2 * (size_t)n_policies * align256(chunk * sizeof(convgpu_summary_t)) +
-         (size_t)n_policies * align256(sizeof(convgpu_stats_t)) + cn;  // + admission scratch
+namespace {
+
+struct HostLayout {
+  size_t cn, ckn, c16n, ck16n, c8n;
+};
+HostLayout host_layout(uint32_t nc, uint32_t K, uint64_t chunk) {
+  HostLayout l;
+  l.cn = align256(chunk * nc * 4);
+  l.ckn = align256(chunk * nc * K * 4);
+  l.c16n = align256(chunk * nc * 2);
+  l.ck16n = align256(chunk * nc * K * 2);
+  l.c8n = align256(chunk * nc);
+  return l;
+}
+size_t host_ws_bytes(bool packed, uint32_t nc, uint32_t K, uint64_t chunk, uint32_t np) {
+  const HostLayout l = host_layout(nc, K, chunk);
+  const size_t in32 = 2 * l.cn + 2 * l.ckn;
+  const size_t in16 = 2 * l.c16n + 2 * l.ck16n + l.c8n;
+  const size_t inputs = packed ? 2 * in16 + in32 : 2 * in32;
+  return inputs + 2 * (size_t)np * align256(chunk * sizeof(convgpu_summary_t)) +
+         (size_t)np * align256(sizeof(convgpu_stats_t)) + l.cn;  // + admission scratch
 }
 
-int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, uint32_t policy_mask,
-                        convgpu_summary_t* host_summary, convgpu_stats_t* host_stats,
-                        void* ws, size_t ws_bytes, uint64_t chunk, void* stream_) {
+// One end-to-end replay from host memory; `t32` or `t16` names the format.
+int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint64_t n, uint32_t cap,
+                uint32_t policy_mask, convgpu_summary_t* host_summary, convgpu_stats_t* host_stats,
+                void* ws, size_t ws_bytes, uint64_t chunk, void* stream_) {
+  const bool packed = t16 != nullptr;
   if (policy_mask == 0 || policy_mask > 0xFu) return -EINVAL;
-  int rc = validate_shape(ht, cap, 0);
+  convgpu_traces_t ht;  // shape / parameters (array pointers unused when packed)
+  if (packed) {
+    memset(&ht, 0, sizeof ht);
+    ht.n_containers = t16->n_containers; ht.n_ops = t16->n_ops;
+    ht.trace_id_base = t16->trace_id_base; ht.rand_seed = t16->rand_seed;
+    ht.ctx_overhead_mib = t16->ctx_overhead_mib; ht.kernel_variant = t16->kernel_variant;
+    if (ht.n_ops > 4) return -EINVAL;  // kinds are one byte per container
+  } else {
+    if (!t32) return -EINVAL;
+    ht = *t32;
+  }
+  int rc = validate_shape(&ht, cap, 0);
   if (rc) return rc;
   if (!host_stats || !ws || chunk == 0) return -EINVAL;
-  if ((rc = validate_arrays(ht))) return rc;
+  if (packed ? (!t16->arrival || !t16->limit || !t16->op_size || !t16->op_delta || !t16->op_kinds)
+             : (rc = validate_arrays(&ht)) != 0)
+    return -EINVAL;
   if ((rc = check_device())) return rc;
   int pols[4], np = 0;
   for (int q = 0; q < 4; ++q)
     if (policy_mask & (1u << q)) pols[np++] = q;
-  const uint32_t nc = ht->n_containers, K = ht->n_ops;
-  if (ws_bytes < convgpu_replay_host_workspace(nc, K, chunk, (uint32_t)np) || !is_device_ptr(ws))
+  const uint32_t nc = ht.n_containers, K = ht.n_ops;
+  if (ws_bytes < host_ws_bytes(packed, nc, K, chunk, (uint32_t)np) || !is_device_ptr(ws))
     return -EINVAL;
   cudaStream_t cs = (cudaStream_t)stream_;
-  const size_t cn = align256(chunk * nc * 4), ckn = align256(chunk * nc * K * 4);
+  const HostLayout l = host_layout(nc, K, chunk);
   const size_t sb = align256(chunk * sizeof(convgpu_summary_t));
   char* w = (char*)ws;
+  // 32-bit chunk sets: [0], [1] (copy-in) or [0] only (unpack target)
   uint32_t *arr[2], *lim[2], *del[2], *arg[2];
-  convgpu_summary_t* sum[2][4];
-  for (int b = 0; b < 2; ++b) {
-    arr[b] = (uint32_t*)w; w += cn;
-    lim[b] = (uint32_t*)w; w += cn;
-    del[b] = (uint32_t*)w; w += ckn;
-    arg[b] = (uint32_t*)w; w += ckn;
+  uint16_t *arr16[2] = {nullptr, nullptr}, *lim16[2] = {nullptr, nullptr};
+  uint16_t *siz16[2] = {nullptr, nullptr}, *del16[2] = {nullptr, nullptr};
+  uint8_t* kin8[2] = {nullptr, nullptr};
+  for (int b = 0; b < (packed ? 1 : 2); ++b) {
+    arr[b] = (uint32_t*)w; w += l.cn;
+    lim[b] = (uint32_t*)w; w += l.cn;
+    del[b] = (uint32_t*)w; w += l.ckn;
+    arg[b] = (uint32_t*)w; w += l.ckn;
   }
+  if (packed) {
+    arr[1] = arr[0]; lim[1] = lim[0]; del[1] = del[0]; arg[1] = arg[0];
+    for (int b = 0; b < 2; ++b) {
+      arr16[b] = (uint16_t*)w; w += l.c16n;
+      lim16[b] = (uint16_t*)w; w += l.c16n;
+      siz16[b] = (uint16_t*)w; w += l.ck16n;
+      del16[b] = (uint16_t*)w; w += l.ck16n;
+      kin8[b] = (uint8_t*)w; w += l.c8n;
+    }
+  }
+  convgpu_summary_t* sum[2][4];
   for (int b = 0; b < 2; ++b)
     for (int q = 0; q < np; ++q) { sum[b][q] = (convgpu_summary_t*)w; w += sb; }
   convgpu_stats_t* dstats = (convgpu_stats_t*)w;  // [np], 256-B apart
@@ -271,11 +319,24 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     const int b = (int)(j & 1);
     const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
     cudaError_t r = cudaSuccess;
-    if (j >= 2) r = cudaStreamWaitEvent(copy, kdone[b], 0);  // buffer b free again
-    if (r == cudaSuccess) r = cudaMemcpyAsync(arr[b], ht->arrival + lo * nc, cnt * nc * 4, cudaMemcpyHostToDevice, copy);
-    if (r == cudaSuccess) r = cudaMemcpyAsync(lim[b], ht->limit + lo * nc, cnt * nc * 4, cudaMemcpyHostToDevice, copy);
-    if (r == cudaSuccess) r = cudaMemcpyAsync(del[b], ht->op_delta + lo * nc * K, cnt * nc * K * 4, cudaMemcpyHostToDevice, copy);
-    if (r == cudaSuccess) r = cudaMemcpyAsync(arg[b], ht->op_arg + lo * nc * K, cnt * nc * K * 4, cudaMemcpyHostToDevice, copy);
+    // copy-in buffer b is free again once the chunk j - 2 that used it is
+    // consumed (replayed; packed: unpacked, ordered before its replays)
+    if (j >= 2) r = cudaStreamWaitEvent(copy, kdone[b], 0);
+    auto cp = [&](void* dst, const void* src, size_t bytes) {
+      if (r == cudaSuccess) r = cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, copy);
+    };
+    if (packed) {
+      cp(arr16[b], t16->arrival + lo * nc, cnt * nc * 2);
+      cp(lim16[b], t16->limit + lo * nc, cnt * nc * 2);
+      cp(siz16[b], t16->op_size + lo * nc * K, cnt * nc * K * 2);
+      cp(del16[b], t16->op_delta + lo * nc * K, cnt * nc * K * 2);
+      cp(kin8[b], t16->op_kinds + lo * nc, cnt * nc);
+    } else {
+      cp(arr[b], ht.arrival + lo * nc, cnt * nc * 4);
+      cp(lim[b], ht.limit + lo * nc, cnt * nc * 4);
+      cp(del[b], ht.op_delta + lo * nc * K, cnt * nc * K * 4);
+      cp(arg[b], ht.op_arg + lo * nc * K, cnt * nc * K * 4);
+    }
     if (r == cudaSuccess) r = cudaEventRecord(h2d[b], copy);
     return r;
   };
@@ -292,15 +353,25 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
     // summary buffers b: read back (chunk j - 2) before they are rewritten
     if (e == cudaSuccess && host_summary && j >= 2) e = cudaStreamWaitEvent(cs, d2h[b], 0);
     if (e != cudaSuccess) break;
-    convgpu_traces_t dt = *ht;
+    if (packed) {  // 16-bit copy-in buffer b -> the 32-bit chunk set
+      convgpu::Pack16Args u;
+      memset(&u, 0, sizeof u);
+      u.count = cnt; u.n = nc; u.K = K;
+      u.r_arrival16 = arr16[b]; u.r_limit16 = lim16[b]; u.r_size16 = siz16[b];
+      u.r_delta16 = del16[b]; u.r_kinds8 = kin8[b];
+      u.w_arrival = arr[b]; u.w_limit = lim[b]; u.w_delta = del[b]; u.w_arg = arg[b];
+      e = convgpu::launch_unpack16(u, cs);
+      if (e != cudaSuccess) break;
+    }
+    convgpu_traces_t dt = ht;
     dt.arrival = arr[b]; dt.limit = lim[b]; dt.op_delta = del[b]; dt.op_arg = arg[b];
-    dt.trace_id_base = ht->trace_id_base + lo;
+    dt.trace_id_base = ht.trace_id_base + lo;
     for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
       a.adm_scratch = adm_scratch;  // admissions only; no per-container outputs
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
-      e = launch_any(a, pols[q], ht->kernel_variant, cs);
+      e = launch_any(a, pols[q], ht.kernel_variant, cs);
     }
     if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
     if (e == cudaSuccess && host_summary) {
@@ -341,6 +412,59 @@ int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, ui
   if (copy) cudaStreamDestroy(copy);
   if (back) cudaStreamDestroy(back);
   return e == cudaSuccess ? 0 : fail_cuda(e, "replay_host");
+}
+
+}  // namespace
+
+size_t convgpu_replay_host_workspace(uint32_t n_containers, uint32_t n_ops, uint64_t chunk,
+                                     uint32_t n_policies) {
+  return host_ws_bytes(false, n_containers, n_ops, chunk, n_policies);
+}
+
+size_t convgpu_replay_host16_workspace(uint32_t n_containers, uint32_t n_ops, uint64_t chunk,
+                                       uint32_t n_policies) {
+  return host_ws_bytes(true, n_containers, n_ops, chunk, n_policies);
+}
+
+int convgpu_replay_host(const convgpu_traces_t* ht, uint64_t n, uint32_t cap, uint32_t policy_mask,
+                        convgpu_summary_t* host_summary, convgpu_stats_t* host_stats,
+                        void* ws, size_t ws_bytes, uint64_t chunk, void* stream_) {
+  if (!ht) return -EINVAL;
+  return host_replay(ht, nullptr, n, cap, policy_mask, host_summary, host_stats, ws, ws_bytes,
+                     chunk, stream_);
+}
+
+int convgpu_replay_host16(const convgpu_traces16_t* ht, uint64_t n, uint32_t cap,
+                          uint32_t policy_mask, convgpu_summary_t* host_summary,
+                          convgpu_stats_t* host_stats, void* ws, size_t ws_bytes, uint64_t chunk,
+                          void* stream_) {
+  if (!ht) return -EINVAL;
+  return host_replay(nullptr, ht, n, cap, policy_mask, host_summary, host_stats, ws, ws_bytes,
+                     chunk, stream_);
+}
+
+int convgpu_pack16(const convgpu_traces_t* src, uint64_t n, const convgpu_trace16_buffers_t* dst,
+                   uint64_t* out_of_range, void* stream) {
+  if (!src || !dst) return -EINVAL;
+  if (src->n_containers < 1 || src->n_containers > CONVGPU_MAX_CONTAINERS) return -EINVAL;
+  if (src->n_ops < 1 || src->n_ops > 4) return -EINVAL;
+  int rc = check_device();
+  if (rc) return rc;
+  if (n == 0) return 0;
+  if (!is_device_ptr(src->arrival) || !is_device_ptr(src->limit) || !is_device_ptr(src->op_delta) ||
+      !is_device_ptr(src->op_arg) || !is_device_ptr(dst->arrival) || !is_device_ptr(dst->limit) ||
+      !is_device_ptr(dst->op_size) || !is_device_ptr(dst->op_delta) ||
+      !is_device_ptr(dst->op_kinds) || !opt_device_ptr(out_of_range))
+    return -EINVAL;
+  convgpu::Pack16Args a;
+  memset(&a, 0, sizeof a);
+  a.count = n; a.n = src->n_containers; a.K = src->n_ops;
+  a.arrival = src->arrival; a.limit = src->limit; a.delta = src->op_delta; a.arg = src->op_arg;
+  a.arrival16 = dst->arrival; a.limit16 = dst->limit; a.size16 = dst->op_size;
+  a.delta16 = dst->op_delta; a.kinds8 = dst->op_kinds;
+  a.out_of_range = (unsigned long long*)out_of_range;
+  cudaError_t e = convgpu::launch_pack16(a, (cudaStream_t)stream);
+  return e == cudaSuccess ? 0 : fail_cuda(e, "pack16 launch");
 }
 
 }  // extern "C"

@@ -50,6 +50,24 @@ struct GenArgs {
 
 cudaError_t launch_generate(const GenArgs& a, cudaStream_t stream);
 
+// pack16.cu: 32-bit SoA <-> compact 16-bit trace format (convgpu_traces16_t)
+struct Pack16Args {
+  uint64_t count;
+  uint32_t n, K;
+  // pack: read 32-bit, write 16-bit
+  const uint32_t *arrival, *limit, *delta, *arg;
+  uint16_t *arrival16, *limit16, *size16, *delta16;
+  uint8_t* kinds8;
+  unsigned long long* out_of_range;  // values that do not fit (accumulated), or NULL
+  // unpack: read 16-bit, write 32-bit
+  const uint16_t *r_arrival16, *r_limit16, *r_size16, *r_delta16;
+  const uint8_t* r_kinds8;
+  uint32_t *w_arrival, *w_limit, *w_delta, *w_arg;
+};
+
+cudaError_t launch_pack16(const Pack16Args& a, cudaStream_t stream);
+cudaError_t launch_unpack16(const Pack16Args& a, cudaStream_t stream);
+
 cudaError_t launch_wrap(const uint4* api, uint64_t count, uint32_t n, uint32_t K, uint32_t pitch,
                         uint32_t* arg, cudaStream_t stream);
 

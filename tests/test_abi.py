@@ -123,3 +123,42 @@ def test_missing_extension_fails_loudly(monkeypatch, tmp_path):
     monkeypatch.setattr(cg, "_lib", None)
     with pytest.raises(cg.ConvgpuError):
         cg.lib()
+
+
+def _traces16(**kw):
+    t = cg.Traces16T(1, 1, 1, 1, 1, 64, 4, 0, 0, 0, 0)
+    for k, v in kw.items():
+        setattr(t, k, v)
+    return t
+
+
+@pytest.mark.parametrize("kw", [dict(n_ops=5), dict(n_ops=0), dict(n_containers=65),
+                                dict(op_kinds=None), dict(arrival=None), dict(kernel_variant=4)])
+def test_replay_host16_rejects_bad_shape_before_touching_the_device(so, kw):
+    st = (C.c_uint8 * 96)()
+    assert so.convgpu_replay_host16(C.byref(_traces16(**kw)), 10, 1000, 1, None, st, 1, 1 << 30,
+                                    16, None) == -errno.EINVAL
+
+
+def test_replay_host16_rejects_empty_mask_and_null(so):
+    st = (C.c_uint8 * 96)()
+    assert so.convgpu_replay_host16(C.byref(_traces16()), 10, 1000, 0, None, st, 1, 1 << 30,
+                                    16, None) == -errno.EINVAL
+    assert so.convgpu_replay_host16(None, 10, 1000, 1, None, st, 1, 1 << 30, 16,
+                                    None) == -errno.EINVAL
+
+
+def test_pack16_rejects_bad_shape(so):
+    buf = cg.Buffers16T(1, 1, 1, 1, 1)
+    assert so.convgpu_pack16(C.byref(_traces(n_ops=5)), 10, C.byref(buf), None, None) == -errno.EINVAL
+    assert so.convgpu_pack16(C.byref(_traces(n_containers=0)), 10, C.byref(buf), None,
+                             None) == -errno.EINVAL
+    assert so.convgpu_pack16(None, 10, C.byref(buf), None, None) == -errno.EINVAL
+
+
+def test_workspace16_size(so):
+    """The 16-bit path holds two 16-bit copy-in sets and one 32-bit unpack
+    target instead of two 32-bit sets."""
+    w32 = so.convgpu_replay_host_workspace(64, 4, 1000, 4)
+    w16 = so.convgpu_replay_host16_workspace(64, 4, 1000, 4)
+    assert w16 >= w32 - 1000 * 64 * 40 + 2 * 1000 * 64 * 21
