@@ -61,7 +61,9 @@ def parse():
     ap.add_argument("--outputs", default="full", choices=["full", "summary"])
     ap.add_argument("--kernel", default="auto", choices=["auto", "warp", "lane", "lane16"])
     ap.add_argument("--e2e-steps", type=int, default=5)
-    ap.add_argument("--e2e-chunk", type=int, default=1 << 15, help="traces per host-path chunk")
+    ap.add_argument("--e2e-chunk", type=int, default=0,
+                    help="traces per host-path chunk (0: one full wave of the compact kernel, "
+                         "SMs x 256 lanes)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-check", action="store_true", help="skip the golden-range parity check")
     ap.add_argument("--c3-chunk", type=int, default=4 << 20, help="traces per chunk (config [3])")
@@ -551,7 +553,7 @@ def run_ours(args, rank, local_rank, world):
     # B per container instead of 40, unpacked on the device), because the
     # 32-bit path is bound by its PCIe copy; the 32-bit path is timed beside it.
     if not args.no_e2e and not args.profile:
-        chunk = args.e2e_chunk
+        chunk = args.e2e_chunk or sms * 256  # one trace per lane of a full grid
         t16, oor = cg.pack16(tr, stream=stream)
         torch.cuda.synchronize()
         packed_ok = int(oor.item()) == 0  # every value fits 16 bits (exact)

@@ -40,7 +40,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     def compile_one(f):
         obj = os.path.join(objdir, f.replace(".cu", ".o"))
-        cmd = [NVCC, *FLAGS, "-c", "-o", obj, os.path.join(CSRC, f)]
+        # CONVGPU_NVCC_DEFS: extra -D flags for A/B builds of kernel variants
+        extra = os.environ.get("CONVGPU_NVCC_DEFS", "").split()
+        cmd = [NVCC, *FLAGS, *extra, "-c", "-o", obj, os.path.join(CSRC, f)]
         r = subprocess.run(cmd, capture_output=True, text=True)
         return obj, cmd, r
 
