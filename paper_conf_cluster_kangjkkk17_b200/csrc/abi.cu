@@ -231,7 +231,8 @@ size_t host_ws_bytes(bool packed, uint32_t nc, uint32_t K, uint64_t chunk, uint3
   const size_t in16 = 2 * l.c16n + 2 * l.ck16n + l.c8n;
   const size_t inputs = packed ? 2 * in16 + in32 : 2 * in32;
   return inputs + 2 * (size_t)np * align256(chunk * sizeof(convgpu_summary_t)) +
-         (size_t)np * align256(sizeof(convgpu_stats_t)) + l.cn;  // + admission scratch
+         (size_t)np * align256(sizeof(convgpu_stats_t)) +
+         (size_t)np * l.cn;  // + admission scratch, one per policy (they run concurrently)
 }
 
 // One end-to-end replay from host memory; `t32` or `t16` names the format.
@@ -294,13 +295,18 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
     for (int q = 0; q < np; ++q) { sum[b][q] = (convgpu_summary_t*)w; w += sb; }
   convgpu_stats_t* dstats = (convgpu_stats_t*)w;  // [np], 256-B apart
   const size_t stb = align256(sizeof(convgpu_stats_t));
-  // per-container admissions of the chunk being replayed: the compact lane
-  // kernel keeps them here during a replay (launches are stream-ordered)
+  // per-container admissions of the chunk being replayed, one plane per
+  // policy: the policies' replays of a chunk run concurrently
   uint32_t* adm_scratch = (uint32_t*)(w + (size_t)np * stb);
 
   // inputs go in on `copy`, summaries come back on `back` (PCIe is full
   // duplex: the read-back of chunk j overlaps the copy-in of chunk j + 2)
   cudaStream_t copy = nullptr, back = nullptr;
+  // the policies of a chunk replay on their own streams, so one launch's
+  // tail (its last, partly filled round of traces) overlaps the next one's
+  // start instead of leaving SMs idle (the chunk is one round of lanes)
+  cudaStream_t ps[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t ready = nullptr, pdone[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t h2d[2] = {nullptr, nullptr}, kdone[2] = {nullptr, nullptr};
   cudaEvent_t d2h[2] = {nullptr, nullptr};
   cudaEvent_t start_ev = nullptr, copy_done = nullptr, back_done = nullptr;
@@ -311,6 +317,11 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&kdone[b], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&d2h[b], cudaEventDisableTiming);
   }
+  for (int q = 0; q < np && e == cudaSuccess; ++q) {
+    e = cudaStreamCreateWithFlags(&ps[q], cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pdone[q], cudaEventDisableTiming);
+  }
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ready, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&copy_done, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&back_done, cudaEventDisableTiming);
@@ -366,13 +377,18 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
     convgpu_traces_t dt = ht;
     dt.arrival = arr[b]; dt.limit = lim[b]; dt.op_delta = del[b]; dt.op_arg = arg[b];
     dt.trace_id_base = ht.trace_id_base + lo;
+    if (e == cudaSuccess) e = cudaEventRecord(ready, cs);
     for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
+      cudaStream_t sq = ps[q];
+      e = cudaStreamWaitEvent(sq, ready, 0);
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
-      a.adm_scratch = adm_scratch;  // admissions only; no per-container outputs
+      a.adm_scratch = adm_scratch + (size_t)q * l.cn / 4;  // admissions only
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
-      e = launch_any(a, pols[q], ht.kernel_variant, cs);
+      if (e == cudaSuccess) e = launch_any(a, pols[q], ht.kernel_variant, sq);
+      if (e == cudaSuccess) e = cudaEventRecord(pdone[q], sq);
     }
+    for (int q = 0; q < np && e == cudaSuccess; ++q) e = cudaStreamWaitEvent(cs, pdone[q], 0);
     if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
     if (e == cudaSuccess && host_summary) {
       e = cudaStreamWaitEvent(back, kdone[b], 0);
@@ -399,8 +415,15 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
     // (secondary errors ignored; the first one is reported)
     if (copy) cudaStreamSynchronize(copy);
     if (back) cudaStreamSynchronize(back);
+    for (int q = 0; q < 4; ++q)
+      if (ps[q]) cudaStreamSynchronize(ps[q]);
     cudaStreamSynchronize(cs);
   }
+  for (int q = 0; q < 4; ++q) {
+    if (ps[q]) cudaStreamDestroy(ps[q]);
+    if (pdone[q]) cudaEventDestroy(pdone[q]);
+  }
+  if (ready) cudaEventDestroy(ready);
   for (int b = 0; b < 2; ++b) {
     if (h2d[b]) cudaEventDestroy(h2d[b]);
     if (kdone[b]) cudaEventDestroy(kdone[b]);
