@@ -54,8 +54,7 @@ int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
   if (t->n_ops < 1 || t->n_ops > CONVGPU_MAX_OPS) return -EINVAL;
   if (policy < 0 || (policy & ~(0xFF | CONVGPU_DISPATCH_LITERAL)) || (policy & 0xFF) > 3)
     return -EINVAL;
-  if ((policy & CONVGPU_DISPATCH_LITERAL) && (t->kernel_variant == CONVGPU_KERNEL_LANE_PER_TRACE ||
-                                               t->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT))
+  if ((policy & CONVGPU_DISPATCH_LITERAL) && t->kernel_variant == CONVGPU_KERNEL_LANE_PER_TRACE)
     return -EINVAL;
   if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
   if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
@@ -102,12 +101,14 @@ uint32_t auto_variant(uint64_t count, int policy) {
 cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cudaStream_t s) {
   a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.adm_scratch) &&
                 aligned16(a.wait) && aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
-  if (policy & CONVGPU_DISPATCH_LITERAL) variant = CONVGPU_KERNEL_WARP_PER_TRACE;
   if (variant == CONVGPU_KERNEL_AUTO) {
     variant = auto_variant(a.count, policy);
     if (variant == CONVGPU_KERNEL_LANE_PER_TRACE && convgpu::lpt16_supported(a))
       variant = CONVGPU_KERNEL_LANE_COMPACT;
   }
+  // R1-LIT runs on the compact kernel or the warp-per-trace kernel
+  if ((policy & CONVGPU_DISPATCH_LITERAL) && variant == CONVGPU_KERNEL_LANE_PER_TRACE)
+    variant = CONVGPU_KERNEL_WARP_PER_TRACE;
   if (variant == CONVGPU_KERNEL_LANE_COMPACT) {
     if (!convgpu::lpt16_supported(a)) return cudaErrorInvalidValue;  // -EINVAL, see convgpu_replay
     return convgpu::launch_replay_lpt16(a, policy, s);

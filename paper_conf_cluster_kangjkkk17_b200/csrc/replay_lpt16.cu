@@ -69,14 +69,19 @@ constexpr uint32_t kTmemCols = 128;
  // 64 per warp, warps w and w + 4 share a lane quarter
 
 // bytes per lane (= per trace) and warps per CTA (one CTA per SM)
+// policy may carry CONVGPU_DISPATCH_LITERAL (R1-LIT, NEXT-1): several
+// containers then hold partial assignments, kept as u16 per container
+__host__ __device__ constexpr bool is_lit(int policy) {
+  return (policy & CONVGPU_DISPATCH_LITERAL) != 0;
+}
 __host__ __device__ constexpr uint32_t extra_bytes(int policy) {
-  return 0u;  // every policy's extra state lives in registers (Best-Fit: limit classes)
+  return is_lit(policy) ? N * 2u : 0u;  // R1: every policy's extra state lives in registers
 }
 __host__ __device__ constexpr uint32_t lane_bytes(int policy) {
   return N * 14u + extra_bytes(policy) + 8u;  // + 2-word fetch staging slot
 }
 __host__ __device__ constexpr int warps_per_cta(int policy) {
-  return 8;
+  return is_lit(policy) ? 7 : 8;  // 1,032 B per trace under R1-LIT
 }
 // Best-Fit keeps the trace's distinct declared limits ("classes") in
 // registers; a trace with more distinct limits than this is left to the
@@ -97,6 +102,8 @@ __device__ __forceinline__ uint32_t pack_sd(uint32_t cw, uint32_t d) {
 template <int POLICY>
 __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
+  constexpr bool LIT = is_lit(POLICY);     // R1-LIT (NEXT-1) instead of R1
+  constexpr int P = POLICY & 0xFF;         // convgpu_policy_t
   const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
   constexpr uint32_t n = N, K = KOPS;
   const uint32_t cap = p.cap, ovh = p.ovh;
@@ -110,9 +117,12 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // address; at most 2-way bank conflicts, between lanes 2j and 2j + 1)
   uint16_t* const s_L = reinterpret_cast<uint16_t*>(W0 + 3 * n * 32) + lane;
   // staging slot of the one-op-ahead fetch: {op word, delta of the op after}
+  // R1-LIT: assignment a of container c (u16, at most its limit), [c][lane]
+  uint16_t* const s_A = reinterpret_cast<uint16_t*>(W0 + (3 * n + n / 2) * 32) + lane;
   uint32_t* const s_stg = W0 + (3 * n + n / 2 + extra_bytes(POLICY) / 4) * 32 + lane;
 #define AT(arr, c) (arr)[(c) * 32u]
 #define LIM(c) s_L[(c) * 32u]
+#define ASG(c) s_A[(c) * 32u]
 
   // A warp replays 32 consecutive traces per round; round-robin warp slots
   // run SM-first (slot = wib * gridDim + block), so the last, partial round
@@ -225,6 +235,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu);
         AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
         LIM(c) = (uint16_t)min(L, 0xFFFFu);
+        if (LIT) ASG(c) = 0;
         gmin[c >> 3] = min(gmin[c >> 3], key);
         base[c] = bsum;
         if (c == 0) arr0 = a;
@@ -238,7 +249,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     // previous call may have left in caller scratch (admissions of container
     // 0 are only read back when it was admitted, so 0 is harmless)
     adm_out[0] = skip ? kLpt16Mark : 0u;
-    if (POLICY == CONVGPU_BEST_FIT) {
+    if (P == CONVGPU_BEST_FIT && !LIT) {
       // distinct limits (unsorted while collected), with member masks
       uint32_t ncls = 0;
 #pragma unroll
@@ -399,9 +410,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
             const bool arr = (ust & kNotArrived) == kNotArrived;
             // ARRIVE (Fig. 3b/3c; R2)
-            const uint32_t g = (arr && target == kNoC) ? min(L, free_mem) : 0u;
+            // R1-LIT: every newcomer takes what is free (no fill target)
+            const uint32_t g = (arr && (LIT || target == kNoC)) ? min(L, free_mem) : 0u;
             const bool vadm = arr && g == L;
-            const bool vtgt = arr && !vadm && g > 0;
+            const bool vtgt = !LIT && arr && !vadm && g > 0;
             // An arrival whose first op has delta 0 (before arrival the used
             // field holds d_0) is followed by that op at the same tick: the
             // DISPATCH after an ARRIVE is empty (with a target free = 0 and the
@@ -423,7 +435,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const bool isF = op && kind == CONVGPU_OP_FREE;
             const bool isX = op && kind == CONVGPU_OP_FINISH;
             const bool tnone = tg1 == kNoC, ctg = c == tg1;
-            const uint32_t a_c = (ust1 & kAdmitted) ? L : (vtgt ? g : (ctg ? a_tg : 0u));
+            const uint32_t a_c =
+                (ust1 & kAdmitted) ? L
+                                   : (LIT ? (arr ? g : (uint32_t)ASG(c)) : (vtgt ? g : (ctg ? a_tg : 0u)));
+            if (LIT && arr) ASG(c) = (uint16_t)g;
             // ALLOC
             const uint32_t need = used + r + ((ust1 & kFirst) ? 0u : ovh);
             const bool rej = isA && need > L;                // R10
@@ -451,9 +466,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             // Recent-Fit: push c on the suspension stack (its key links the old
             // top) unless it is the fill target, which resumes without a
             // selection (R1) and so must never be popped
-            const uint32_t plink = (POLICY == CONVGPU_RECENT_FIT) ? ru_head : 0u;
-            if (POLICY == CONVGPU_RECENT_FIT) ru_head = (pause && !ctg) ? c : ru_head;
-            dmode = (pause & tnone) | (isX & ((target != kNoC) | ((pm_lo | pm_hi) != 0u)));
+            const uint32_t plink = (P == CONVGPU_RECENT_FIT) ? ru_head : 0u;
+            if (P == CONVGPU_RECENT_FIT) ru_head = (pause && !ctg) ? c : ru_head;
+            // R1-LIT dispatches whenever memory is free and someone is paused
+            dmode = LIT ? (free_mem != 0u && (pm_lo | pm_hi) != 0u)
+                        : (pause & tnone) | (isX & ((target != kNoC) | ((pm_lo | pm_hi) != 0u)));
             if (badfree) { flags |= CONVGPU_FLAG_INVALID_FREE; tdone = true;
 #ifdef LPT16_DEBUG
               dbg0 = c | (k << 8) | ((uint32_t)(pre_c) << 16); dbg1 = r; dbg2 = used; dbg3 = ust; dbg4 = sd;
@@ -474,15 +491,31 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         } else if (dmode) {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
           const uint32_t t = cur_t;
-          if (POLICY == CONVGPU_FIFO) {
-            const bool ns = target == kNoC;
+          if (P == CONVGPU_FIFO) {
+            const bool ns = target == kNoC;  // (always under R1-LIT: no sticky target)
             const uint32_t sel = ffs64(pm_lo, pm_hi);
             target = ns ? sel : target;
             a_tg = ns ? 0u : a_tg;
             n_sel += ns ? 1u : 0u;
           } else if (target == kNoC) {
             uint32_t sel;
-            if (POLICY == CONVGPU_BEST_FIT) {  // R3, R4 (classes: see bl above)
+            if (P == CONVGPU_BEST_FIT && LIT) {  // R3, R4 with partial holds: shortfall L - a
+              uint32_t best = kNoC, bneed = 0, mn = kNoC, mneed = 0xFFFFFFFFu;
+              uint32_t wl = pm_lo, wh = pm_hi;
+              while (wl | wh) {  // ascending index: strict comparisons keep the lowest
+                const uint32_t c = ffs64(wl, wh);
+                wl &= ~shl_c(1u, c);
+                wh &= ~shl_c(1u, c - 32u);
+                const uint32_t need = (uint32_t)LIM(c) - (uint32_t)ASG(c);
+                const bool f = need <= free_mem && (best == kNoC || need > bneed);
+                best = f ? c : best;
+                bneed = f ? need : bneed;
+                const bool m = need < mneed;
+                mn = m ? c : mn;
+                mneed = m ? need : mneed;
+              }
+              sel = best != kNoC ? best : mn;
+            } else if (P == CONVGPU_BEST_FIT) {  // R3, R4 (classes: see bl above)
               // ascending classes: the last fitting class with a paused
               // member wins; descending: the last class with one is the lowest
               uint32_t fl = 0, fh = 0, ml = 0, mh = 0;
@@ -502,13 +535,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
               }
               const bool fit = (fl | fh) != 0u;
               sel = ffs64(fit ? fl : ml, fit ? fh : mh);
-            } else if (POLICY == CONVGPU_RECENT_FIT) {  // R5
+            } else if (P == CONVGPU_RECENT_FIT) {  // R5
               // pop the suspension stack: paused containers leave the paused
               // set only by resuming, and only the target resumes, so popping
               // at selection keeps the stack exactly the paused set in
-              // suspension order
+              // suspension order.  R1-LIT: the selected container may stay
+              // paused (partially filled), so it is popped when it resumes
               sel = ru_head;
-              ru_head = AT(s_key, sel) & 127u;
+              if (!LIT) ru_head = AT(s_key, sel) & 127u;
             } else {  // RANDOM_FIT (R6)
               const uint64_t tid = p.tid_base + i;
               const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
@@ -519,7 +553,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
               sel = lpt::nth_set64(pm_lo, pm_hi, jj);
             }
             target = sel;
-            a_tg = 0;
+            a_tg = LIT ? (uint32_t)ASG(sel) : 0u;  // R1-LIT: its partial hold
             ++n_sel;
           }
           {
@@ -547,9 +581,17 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             pm_hi &= ~(shl_c(1u, tg - 32u) & rmask);
             stg_if(adm_out + tg, (t << 6) | rank, full);
             rank += full ? 1u : 0u;
-            target = full ? kNoC : target;
-            a_tg = full ? 0u : a_tg;
-            dmode = full && (pm_lo | pm_hi) != 0u;
+            if (LIT) {  // no sticky target: select again while memory is free
+              ASG(tg) = (uint16_t)a_tg;
+              if (P == CONVGPU_RECENT_FIT) ru_head = res ? (AT(s_key, tg) & 127u) : ru_head;
+              target = kNoC;
+              a_tg = 0;
+              dmode = free_mem != 0u && (pm_lo | pm_hi) != 0u;
+            } else {
+              target = full ? kNoC : target;
+              a_tg = full ? 0u : a_tg;
+              dmode = full && (pm_lo | pm_hi) != 0u;
+            }
             kc = res ? tg : kNoC;
             nkc = ((t + (sdt >> 16)) << 6) | tg;
             pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
@@ -583,6 +625,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     }
     park_base();
   }
+#undef ASG
 #undef LIM
 #undef AT
 
@@ -657,18 +700,25 @@ bool lpt16_supported(const ReplayArgs& a) {
 
 cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream) {
   cudaError_t e;
-  switch (policy) {
+  const bool lit = (policy & CONVGPU_DISPATCH_LITERAL) != 0;
+  constexpr int L = CONVGPU_DISPATCH_LITERAL;
+  switch ((policy & 0xFF) | (lit ? L : 0)) {
     case CONVGPU_FIFO: e = lpt16::launch_t<CONVGPU_FIFO>(a, stream); break;
     case CONVGPU_BEST_FIT: e = lpt16::launch_t<CONVGPU_BEST_FIT>(a, stream); break;
     case CONVGPU_RECENT_FIT: e = lpt16::launch_t<CONVGPU_RECENT_FIT>(a, stream); break;
     case CONVGPU_RANDOM_FIT: e = lpt16::launch_t<CONVGPU_RANDOM_FIT>(a, stream); break;
+    case CONVGPU_FIFO | L: e = lpt16::launch_t<CONVGPU_FIFO | L>(a, stream); break;
+    case CONVGPU_BEST_FIT | L: e = lpt16::launch_t<CONVGPU_BEST_FIT | L>(a, stream); break;
+    case CONVGPU_RECENT_FIT | L: e = lpt16::launch_t<CONVGPU_RECENT_FIT | L>(a, stream); break;
+    case CONVGPU_RANDOM_FIT | L: e = lpt16::launch_t<CONVGPU_RANDOM_FIT | L>(a, stream); break;
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
   // traces the 16-bit layout cannot hold: the 32-bit lane kernel, marked only
+  // (R1-LIT: the warp-per-trace kernel, which implements that reading)
   ReplayArgs b = a;
   b.only_marked = 1;
-  return launch_replay_lpt(b, policy, stream);
+  return lit ? launch_replay(b, policy, false, stream) : launch_replay_lpt(b, policy, stream);
 }
 
 }  // namespace convgpu

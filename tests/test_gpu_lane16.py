@@ -134,8 +134,8 @@ def test_lane16_rejects_unsupported_shapes(cg):
     with pytest.raises(cg.ConvgpuError):  # neither admit_tick nor the admission scratch
         cg.replay(tr, w2.cap, "fifo", cg.alloc_out(64, 64, full=False, scratch=False),
                   kernel="lane16")
-    with pytest.raises(cg.ConvgpuError):  # R1-LIT runs on the warp kernel only
-        cg.replay(tr, w2.cap, "fifo+literal", cg.alloc_out(64, 64), kernel="lane16")
+    with pytest.raises(cg.ConvgpuError):  # R1-LIT is not on the 32-bit lane kernel
+        cg.replay(tr, w2.cap, "fifo+literal", cg.alloc_out(64, 64), kernel="lane")
 
 
 def _fused_arrival_batch(seed, count, cap, ovh):
@@ -283,3 +283,69 @@ def test_lane16_few_distinct_limits(cg, orc, policy, case):
     _compare_stats(cg, out, ref["stats"])
     if mode in ("valid", "delayed", "over"):
         assert int(ref["stats"]["n_select"]) > 0
+
+
+# ---------------------------------------------------------------- NEXT-1 on the compact kernel
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("rho", [2, 5, 8])
+def test_lane16_literal_rho_sweep(cg, orc, policy, rho):
+    """R1-LIT (literal re-select-on-every-release, partial holds kept) on the
+    compact kernel against the oracle on config [4] traces, element by
+    element, including the traces it deadlocks (rho 5: a few; rho = 8: limits
+    above 16 bits, so every trace takes the warp-kernel fallback pass)."""
+    w = W.rho_sweep(rho, rand_seed=rho + 3)
+    pid = POLS.index(policy) | 0x100
+    ref = orc.replay_range(w, pid, 20_000, 21_500, full=True)
+    tr = cg.generate(w.gen, 20_000, 1_500)
+    out = _gpu_replay(cg, tr, w.cap, policy + "+literal", seed=w.rand_seed, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    out2 = _gpu_replay(cg, tr, w.cap, policy + "+literal", seed=w.rand_seed, full=False,
+                       kernel="lane16")
+    _compare(cg, out2, ref, full=False)
+
+
+LIT_EDGE = [  # (cap, ovh, mode, count)
+    (256, 0, "valid", 700),
+    (300, 5, "mixed", 900),
+    (128, 0, "over", 500),
+    (200, 1, "delayed", 500),
+    (512, 66, "valid", 500),
+]
+
+
+@pytest.mark.parametrize("case", LIT_EDGE, ids=lambda c: f"{c[2]}{c[0]}o{c[1]}")
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_literal_edge_batches(cg, orc, policy, case):
+    """R1-LIT on edge-case programs (delayed first ops, rejections, invalid
+    frees, bad programs, same-tick arrivals) with dense contention, so many
+    containers hold partial assignments and some traces deadlock."""
+    cap, ovh, mode, count = case
+    b = W.random_batch(8800 + cap, count, 64, 4, cap, ovh=ovh, mode=mode, max_arrival_step=1,
+                       limit_choices=range(1, cap + 1))
+    pid = POLS.index(policy) | 0x100
+    base = 55_000_000 + cap
+    ref = orc.replay_batch(b, cap, pid, tid_base=base, rand_seed=6, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=base)
+    out = _gpu_replay(cg, tr, cap, policy + "+literal", seed=6, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    if mode == "valid":
+        assert ref["stats"]["flag_count"][0] > 0  # the literal reading does deadlock here
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_literal_mixed_fallback(cg, orc, policy):
+    """A batch mixing compact-eligible traces with traces whose values exceed
+    the 16-bit fields: the latter are replayed by the warp-per-trace kernel's
+    marked-only pass under R1-LIT; every trace against the oracle."""
+    xb, cap, ovh = _extreme_batch(97, 300, 64, 4)
+    sb = W.random_batch(98, 300, 64, 4, 16, ovh=1, mode="mixed", limit_choices=range(1, 17))
+    mix = W.Batch(64, 4, *(np.concatenate([getattr(sb, f), getattr(xb, f)])[np.argsort(
+        np.arange(600) % 5, kind="stable")] for f in ("arrival", "limit", "delta", "arg")))
+    pid = POLS.index(policy) | 0x100
+    ref = orc.replay_batch(mix, cap, pid, tid_base=31, rand_seed=7, ovh=ovh)
+    tr = cg.traces_from_numpy(mix.arrival, mix.limit, mix.delta, mix.arg, trace_id_base=31)
+    out = _gpu_replay(cg, tr, cap, policy + "+literal", seed=7, ovh=ovh, kernel="lane16")
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
