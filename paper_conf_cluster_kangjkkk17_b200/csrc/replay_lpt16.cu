@@ -495,7 +495,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             const bool ns = target == kNoC;  // (always under R1-LIT: no sticky target)
             const uint32_t sel = ffs64(pm_lo, pm_hi);
             target = ns ? sel : target;
-            a_tg = ns ? 0u : a_tg;
+            a_tg = ns ? (LIT ? (uint32_t)ASG(sel & 63u) : 0u) : a_tg;  // R1-LIT: its partial hold
             n_sel += ns ? 1u : 0u;
           } else if (target == kNoC) {
             uint32_t sel;
