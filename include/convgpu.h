@@ -56,7 +56,9 @@ typedef enum {
  * re-select-on-every-release reading (R1-LIT, SURVEY §8(f)
  * NEXT-1) instead of R1's sticky fill target.  Partial holds are kept, so
  * deadlocks can occur and are reported by CONVGPU_FLAG_DEADLOCK.  Runs on the
- * warp-per-trace kernel (AUTO selects it; LANE_PER_TRACE is -EINVAL). */
+ * compact lane kernel (AUTO picks it under the same conditions as for R1;
+ * traces it cannot hold go to a marked-only pass of the warp-per-trace
+ * kernel) or on the warp-per-trace kernel; LANE_PER_TRACE is -EINVAL. */
 #define CONVGPU_DISPATCH_LITERAL 0x100
 
 /* Op kinds: op_arg = kind << 30 | size_mib (size < 2^30).  The replay maps
