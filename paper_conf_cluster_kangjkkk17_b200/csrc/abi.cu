@@ -203,13 +203,11 @@ int convgpu_wrap_ops(const convgpu_api_op_t* api, uint64_t n, uint32_t n_contain
 }
 
 // ---------------------------------------------------------------- host e2e
-// Workspace layout (256-B aligned pieces).  32-bit format: 2 x {arrival,
-// limit, delta, arg} chunk buffers (double-buffered copy-in).  16-bit format:
-// 2 x {arrival16, limit16, size16, delta16, kinds8} copy-in buffers and one
-// 32-bit chunk set the unpack kernel writes (the replays of chunk j and the
-// unpack of chunk j + 1 are ordered on the caller's stream).  Then 2 x
-// n_policies summary chunks, n_policies stats structs and one chunk of
-// per-container admission scratch.
+// Workspace layout (256-B aligned pieces): 2 x {arrival, limit, delta, arg}
+// 32-bit chunk sets (the copy-in target, or for the 16-bit format the unpack
+// target, which is then copied into 2 x {arrival16, limit16, size16, delta16,
+// kinds8}), 2 x n_policies summary chunks, n_policies stats structs and
+// n_policies chunks of per-container admission scratch.
 static size_t align256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 namespace {
@@ -230,7 +228,7 @@ size_t host_ws_bytes(bool packed, uint32_t nc, uint32_t K, uint64_t chunk, uint3
   const HostLayout l = host_layout(nc, K, chunk);
   const size_t in32 = 2 * l.cn + 2 * l.ckn;
   const size_t in16 = 2 * l.c16n + 2 * l.ck16n + l.c8n;
-  const size_t inputs = packed ? 2 * in16 + in32 : 2 * in32;
+  const size_t inputs = packed ? 2 * in16 + 2 * in32 : 2 * in32;
   return inputs + 2 * (size_t)np * align256(chunk * sizeof(convgpu_summary_t)) +
          (size_t)np * align256(sizeof(convgpu_stats_t)) +
          (size_t)np * l.cn;  // + admission scratch, one per policy (they run concurrently)
@@ -270,19 +268,19 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
   const HostLayout l = host_layout(nc, K, chunk);
   const size_t sb = align256(chunk * sizeof(convgpu_summary_t));
   char* w = (char*)ws;
-  // 32-bit chunk sets: [0], [1] (copy-in) or [0] only (unpack target)
+  // two 32-bit chunk sets (the copy-in target, or the unpack target of the
+  // 16-bit format) and, for the 16-bit format, two 16-bit copy-in sets
   uint32_t *arr[2], *lim[2], *del[2], *arg[2];
   uint16_t *arr16[2] = {nullptr, nullptr}, *lim16[2] = {nullptr, nullptr};
   uint16_t *siz16[2] = {nullptr, nullptr}, *del16[2] = {nullptr, nullptr};
   uint8_t* kin8[2] = {nullptr, nullptr};
-  for (int b = 0; b < (packed ? 1 : 2); ++b) {
+  for (int b = 0; b < 2; ++b) {
     arr[b] = (uint32_t*)w; w += l.cn;
     lim[b] = (uint32_t*)w; w += l.cn;
     del[b] = (uint32_t*)w; w += l.ckn;
     arg[b] = (uint32_t*)w; w += l.ckn;
   }
-  if (packed) {
-    arr[1] = arr[0]; lim[1] = lim[0]; del[1] = del[0]; arg[1] = arg[0];
+  if (packed)
     for (int b = 0; b < 2; ++b) {
       arr16[b] = (uint16_t*)w; w += l.c16n;
       lim16[b] = (uint16_t*)w; w += l.c16n;
@@ -290,50 +288,49 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
       del16[b] = (uint16_t*)w; w += l.ck16n;
       kin8[b] = (uint8_t*)w; w += l.c8n;
     }
-  }
   convgpu_summary_t* sum[2][4];
   for (int b = 0; b < 2; ++b)
     for (int q = 0; q < np; ++q) { sum[b][q] = (convgpu_summary_t*)w; w += sb; }
   convgpu_stats_t* dstats = (convgpu_stats_t*)w;  // [np], 256-B apart
   const size_t stb = align256(sizeof(convgpu_stats_t));
-  // per-container admissions of the chunk being replayed, one plane per
-  // policy: the policies' replays of a chunk run concurrently
+  // per-container admissions, one plane per policy (each policy replays its
+  // chunks in order on its own stream)
   uint32_t* adm_scratch = (uint32_t*)(w + (size_t)np * stb);
 
-  // inputs go in on `copy`, summaries come back on `back` (PCIe is full
-  // duplex: the read-back of chunk j overlaps the copy-in of chunk j + 2)
+  // Pipeline (b = chunk j & 1):
+  //   copy:  [in-buffer b free] H2D chunk j -> h2d[b]
+  //   cs:    wait h2d[b] (16-bit: [32-bit set b free] unpack -> unp[b]) -> ready[b]
+  //   ps[q]: wait ready[b] [summaries b read back] replay policy q -> pdone[q]
+  //   back:  wait every pdone -> kdone[b] (set b free), D2H summaries -> d2h[b]
+  // Every policy has its own stream, and a policy's chunk j + 1 does not wait
+  // for the other policies' chunk j: the tail of one launch (its last, partly
+  // filled round of lanes) overlaps the start of the next.  PCIe is full
+  // duplex: read-backs overlap copy-ins.
   cudaStream_t copy = nullptr, back = nullptr;
-  // the policies of a chunk replay on their own streams, so one launch's
-  // tail (its last, partly filled round of traces) overlaps the next one's
-  // start instead of leaving SMs idle (the chunk is one round of lanes)
   cudaStream_t ps[4] = {nullptr, nullptr, nullptr, nullptr};
-  cudaEvent_t ready = nullptr, pdone[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t pdone[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t h2d[2] = {nullptr, nullptr}, kdone[2] = {nullptr, nullptr};
-  cudaEvent_t d2h[2] = {nullptr, nullptr};
-  cudaEvent_t start_ev = nullptr, copy_done = nullptr, back_done = nullptr;
+  cudaEvent_t d2h[2] = {nullptr, nullptr}, ready[2] = {nullptr, nullptr}, unp[2] = {nullptr, nullptr};
+  cudaEvent_t start_ev = nullptr;
   cudaError_t e = cudaStreamCreateWithFlags(&copy, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&back, cudaStreamNonBlocking);
-  for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
-    e = cudaEventCreateWithFlags(&h2d[b], cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&kdone[b], cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&d2h[b], cudaEventDisableTiming);
-  }
+  auto mk = [&](cudaEvent_t* ev) {
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(ev, cudaEventDisableTiming);
+  };
+  for (int b = 0; b < 2; ++b) { mk(&h2d[b]); mk(&kdone[b]); mk(&d2h[b]); mk(&ready[b]); mk(&unp[b]); }
   for (int q = 0; q < np && e == cudaSuccess; ++q) {
     e = cudaStreamCreateWithFlags(&ps[q], cudaStreamNonBlocking);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pdone[q], cudaEventDisableTiming);
+    mk(&pdone[q]);
   }
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ready, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&start_ev, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&copy_done, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&back_done, cudaEventDisableTiming);
+  mk(&start_ev);
   const uint64_t nchunks = (n + chunk - 1) / chunk;
   auto enqueue_h2d = [&](uint64_t j) -> cudaError_t {
     const int b = (int)(j & 1);
     const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
     cudaError_t r = cudaSuccess;
-    // copy-in buffer b is free again once the chunk j - 2 that used it is
-    // consumed (replayed; packed: unpacked, ordered before its replays)
-    if (j >= 2) r = cudaStreamWaitEvent(copy, kdone[b], 0);
+    // copy-in buffer b is free again once chunk j - 2 is consumed: unpacked
+    // (16-bit) or replayed by every policy (32-bit)
+    if (j >= 2) r = cudaStreamWaitEvent(copy, packed ? unp[b] : kdone[b], 0);
     auto cp = [&](void* dst, const void* src, size_t bytes) {
       if (r == cudaSuccess) r = cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, copy);
     };
@@ -354,60 +351,65 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
   };
   for (int q = 0; q < np && e == cudaSuccess; ++q)
     e = cudaMemsetAsync((char*)dstats + q * stb, 0, sizeof(convgpu_stats_t), cs);
-  if (e == cudaSuccess) e = cudaEventRecord(start_ev, cs);
+  if (e == cudaSuccess) e = cudaEventRecord(start_ev, cs);  // stats zeroed; the call starts
   if (e == cudaSuccess) e = cudaStreamWaitEvent(copy, start_ev, 0);
+  for (int q = 0; q < np && e == cudaSuccess; ++q) e = cudaStreamWaitEvent(ps[q], start_ev, 0);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(back, start_ev, 0);
   if (e == cudaSuccess && nchunks) e = enqueue_h2d(0);
   for (uint64_t j = 0; j < nchunks && e == cudaSuccess; ++j) {
     const int b = (int)(j & 1);
     const uint64_t lo = j * chunk, cnt = (n - lo < chunk) ? n - lo : chunk;
     if (j + 1 < nchunks) e = enqueue_h2d(j + 1);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, h2d[b], 0);
-    // summary buffers b: read back (chunk j - 2) before they are rewritten
-    if (e == cudaSuccess && host_summary && j >= 2) e = cudaStreamWaitEvent(cs, d2h[b], 0);
-    if (e != cudaSuccess) break;
-    if (packed) {  // 16-bit copy-in buffer b -> the 32-bit chunk set
+    if (packed && e == cudaSuccess) {  // 16-bit copy-in set b -> 32-bit set b
+      if (j >= 2) e = cudaStreamWaitEvent(cs, kdone[b], 0);
       convgpu::Pack16Args u;
       memset(&u, 0, sizeof u);
       u.count = cnt; u.n = nc; u.K = K;
       u.r_arrival16 = arr16[b]; u.r_limit16 = lim16[b]; u.r_size16 = siz16[b];
       u.r_delta16 = del16[b]; u.r_kinds8 = kin8[b];
       u.w_arrival = arr[b]; u.w_limit = lim[b]; u.w_delta = del[b]; u.w_arg = arg[b];
-      e = convgpu::launch_unpack16(u, cs);
-      if (e != cudaSuccess) break;
+      if (e == cudaSuccess) e = convgpu::launch_unpack16(u, cs);
+      if (e == cudaSuccess) e = cudaEventRecord(unp[b], cs);
     }
+    if (e == cudaSuccess) e = cudaEventRecord(ready[b], cs);
+    if (e != cudaSuccess) break;
     convgpu_traces_t dt = ht;
     dt.arrival = arr[b]; dt.limit = lim[b]; dt.op_delta = del[b]; dt.op_arg = arg[b];
     dt.trace_id_base = ht.trace_id_base + lo;
-    if (e == cudaSuccess) e = cudaEventRecord(ready, cs);
     for (int q = 0; q < np && e == cudaSuccess; ++q) {  // every policy on the resident chunk
-      cudaStream_t sq = ps[q];
-      e = cudaStreamWaitEvent(sq, ready, 0);
+      e = cudaStreamWaitEvent(ps[q], ready[b], 0);
+      // summary buffers b: read back (chunk j - 2) before they are rewritten
+      if (e == cudaSuccess && host_summary && j >= 2) e = cudaStreamWaitEvent(ps[q], d2h[b], 0);
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
       a.adm_scratch = adm_scratch + (size_t)q * l.cn / 4;  // admissions only
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
-      if (e == cudaSuccess) e = launch_any(a, pols[q], ht.kernel_variant, sq);
-      if (e == cudaSuccess) e = cudaEventRecord(pdone[q], sq);
+      if (e == cudaSuccess) e = launch_any(a, pols[q], ht.kernel_variant, ps[q]);
+      if (e == cudaSuccess) e = cudaEventRecord(pdone[q], ps[q]);
+      if (e == cudaSuccess) e = cudaStreamWaitEvent(back, pdone[q], 0);
     }
-    for (int q = 0; q < np && e == cudaSuccess; ++q) e = cudaStreamWaitEvent(cs, pdone[q], 0);
-    if (e == cudaSuccess) e = cudaEventRecord(kdone[b], cs);
+    if (e == cudaSuccess) e = cudaEventRecord(kdone[b], back);
     if (e == cudaSuccess && host_summary) {
-      e = cudaStreamWaitEvent(back, kdone[b], 0);
       for (int q = 0; q < np && e == cudaSuccess; ++q)
         e = cudaMemcpyAsync(host_summary + (uint64_t)q * n + lo, sum[b][q],
                             cnt * sizeof(convgpu_summary_t), cudaMemcpyDeviceToHost, back);
       if (e == cudaSuccess) e = cudaEventRecord(d2h[b], back);
     }
   }
+  // join every internal stream back into the caller's stream (events on
+  // `stream` then bracket every copy and kernel of the call), then the stats
+  for (int q = 0; q < np && e == cudaSuccess; ++q) {
+    e = cudaEventRecord(pdone[q], ps[q]);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, pdone[q], 0);
+  }
+  if (e == cudaSuccess) e = cudaEventRecord(h2d[0], copy);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, h2d[0], 0);
+  if (e == cudaSuccess) e = cudaEventRecord(d2h[0], back);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, d2h[0], 0);
   for (int q = 0; q < np && e == cudaSuccess; ++q)
     e = cudaMemcpyAsync(host_stats + q, (char*)dstats + q * stb, sizeof(convgpu_stats_t),
                         cudaMemcpyDeviceToHost, cs);
-  // join the copy stream back into the caller's stream (events on `stream`
-  // then bracket every copy and kernel of the call)
-  if (e == cudaSuccess) e = cudaEventRecord(copy_done, copy);
-  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, copy_done, 0);
-  if (e == cudaSuccess) e = cudaEventRecord(back_done, back);
-  if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, back_done, 0);
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
   if (e != cudaSuccess) {
     // an error mid-way: copies and kernels already enqueued may still read the
@@ -420,19 +422,16 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
       if (ps[q]) cudaStreamSynchronize(ps[q]);
     cudaStreamSynchronize(cs);
   }
+  for (int b = 0; b < 2; ++b) {
+    cudaEvent_t* evs[] = {&h2d[b], &kdone[b], &d2h[b], &ready[b], &unp[b]};
+    for (cudaEvent_t* ev : evs)
+      if (*ev) cudaEventDestroy(*ev);
+  }
   for (int q = 0; q < 4; ++q) {
     if (ps[q]) cudaStreamDestroy(ps[q]);
     if (pdone[q]) cudaEventDestroy(pdone[q]);
   }
-  if (ready) cudaEventDestroy(ready);
-  for (int b = 0; b < 2; ++b) {
-    if (h2d[b]) cudaEventDestroy(h2d[b]);
-    if (kdone[b]) cudaEventDestroy(kdone[b]);
-    if (d2h[b]) cudaEventDestroy(d2h[b]);
-  }
   if (start_ev) cudaEventDestroy(start_ev);
-  if (copy_done) cudaEventDestroy(copy_done);
-  if (back_done) cudaEventDestroy(back_done);
   if (copy) cudaStreamDestroy(copy);
   if (back) cudaStreamDestroy(back);
   return e == cudaSuccess ? 0 : fail_cuda(e, "replay_host");
