@@ -514,6 +514,9 @@ def run_ours(args, rank, local_rank, world):
         issue = {"bound": "alu", "achieved": inst / t_s, "peak": peak_issue, "unit": "warp-inst/s",
                  "frac": inst / t_s / peak_issue,
                  "alu_pipe_pct": {p: ipe[p].get("alu_pipe_pct") for p in POLICIES},
+                 "warp_execution_efficiency": {p: (ipe[p].get("active_lanes") or 0) / 32.0
+                                               for p in POLICIES},
+                 "issue_active_pct_ncu": {p: ipe[p].get("issue_active_pct") for p in POLICIES},
                  "source": "ncu warp instructions per event (" + str(ncu.get("source")) + ") x live "
                            "launch times; peak = SMs x 4 schedulers x 1 instr/clk x SM clock under load"}
 

@@ -42,6 +42,26 @@ b = W.random_batch(6, 300, 64, 4, 64, ovh=1, mode="mixed", limit_choices=range(0
 tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
 for pol in W.POLICIES:
     cg.replay(tr, 64, pol, cg.alloc_out(300, 64), ovh=1, kernel="lane16")
+    # R1-LIT on the compact kernel (+ the warp kernel's marked-only pass) and
+    # summary-only launches through the admission scratch (round 2)
+    cg.replay(tr, 64, pol + "+literal", cg.alloc_out(300, 64), ovh=1, kernel="lane16")
+    cg.replay(tr, 64, pol, cg.alloc_out(300, 64, full=False), ovh=1, kernel="lane16")
+# Best-Fit limit classes: <= 8 distinct limits stay on the compact kernel
+b8 = W.random_batch(7, 300, 64, 4, 256, mode="valid", limit_choices=[0, 13, 62, 105, 148, 165, 201, 256])
+tr8 = cg.traces_from_numpy(b8.arrival, b8.limit, b8.delta, b8.arg)
+cg.replay(tr8, 256, "best_fit", cg.alloc_out(300, 64), kernel="lane16")
+w4 = W.rho_sweep(8, rand_seed=3)
+tr4 = cg.generate(w4.gen, 0, 300)
+for pol in W.POLICIES:
+    cg.replay(tr4, w4.cap, pol + "+literal", cg.alloc_out(300, 64), rand_seed=3, kernel="lane16")
+torch.cuda.synchronize()
+# the 16-bit host format: device packer, host path with the unpack kernel
+w2 = W.CONFIGS["c2"]
+g2 = cg.generate(w2.gen, 0, 20_000)
+t16, oor = cg.pack16(g2)
+h16 = t16.pin()
+summ16 = np.zeros((4, 20_000), cg.SUMMARY_DTYPE)
+cg.replay_host16(h16, w2.cap, W.POLICIES, chunk=9_000, summary=summ16, rand_seed=3)
 torch.cuda.synchronize()
 # the host-memory path (two copy streams, double-buffered chunks, AUTO kernel)
 w = W.CONFIGS["c2"]
