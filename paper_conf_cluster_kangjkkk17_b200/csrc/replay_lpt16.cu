@@ -15,8 +15,15 @@
 //    container's key is 0xC0000000 (Recent-Fit: | the next container down the
 //    suspension stack, which is thereby a linked list needing no extra
 //    memory), both above every event key (ticks < 2^25 here);
-//  * Best-Fit keeps two bytes per container (rank of (L, index), container of
-//    rank) and the "same limit as the previous rank" bits in two registers;
+//  * Best-Fit keeps the trace's distinct limits (at most 8, sorted) and one
+//    64-bit member mask per limit in registers (no shared-memory tables, so
+//    it runs 8 warps per SM too); traces with more distinct limits are left
+//    to the fallback pass;
+//  * arrival + sum of deltas of every container (for R17's wait) is parked
+//    in the thread's tensor-memory lane between init and epilogue;
+//  * under R1-LIT (policy | CONVGPU_DISPATCH_LITERAL, NEXT-1) each
+//    container's partial assignment is a u16 at [container][lane] (7 warps
+//    per SM) and the fallback pass is the warp-per-trace kernel;
 //  * an arrival whose first op has delta 0 is applied together with that op
 //    in one step (see the EVENT step);
 //  * the one-op-ahead fetch (raw op word + next delta, cp.async) lands in a
@@ -24,7 +31,7 @@
 //    end of the NEXT iteration, so the copy has a whole iteration to land
 //    (a register destination would make the compiler wait for it at the loop
 //    head); an event of the container fetched in the previous iteration
-//    (rare) takes a warp-uniform slow path.
+//    (rare) waits one iteration, until the retire has landed its op.
 // A trace qualifies when every limit is <= 0xFFFE MiB, every delta <= 0xFFFF
 // ticks and its horizon (R19) < 2^25 (BASELINE configs [1]-[4] all do; the
 // 16-bit fields are then exact: a saturated size is above every limit, so it
