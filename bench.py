@@ -539,6 +539,7 @@ def run_ours(args, rank, local_rank, world):
                        "parallelism": f"dp{world} (trace-id shards, NCCL stats all-reduce)"},
             "per_policy": {p: {"events_per_s": Nr * per_trace_events * world / (launch_ms[p] / 1e3),
                                "launch_ms": launch_ms[p], "kernel": kernel_of(p),
+                               "hbm_frac": bytes_per_launch / (launch_ms[p] / 1e3) / 1e9 / peak,
                                "digest_sum": "%016x" % (checks[p]["digest_sum"] & (2**64 - 1)),
                                "sum_wait": checks[p]["sum_wait"],
                                "sum_makespan": checks[p]["sum_makespan"]} for p in POLICIES},
