@@ -113,3 +113,30 @@ def test_replay_host16_edge_batches(cg, orc, policy):
         np.testing.assert_array_equal(summ[0][f], ref[f].astype(summ[0][f].dtype), err_msg=f)
     for k, v in ref["stats"].items():
         assert cg.stats_dict(st[0])[k] == v, (policy, k)
+
+
+@pytest.mark.parametrize("policy", ["fifo", "best_fit", "recent_fit", "random_fit"])
+def test_replay_host16_other_shapes(cg, orc, policy):
+    """The 16-bit host path with K = 2 (paper-mimic, n = 38, 66-MiB context)
+    and K = 1 (FINISH-only programs, n = 5): summaries and stats vs the
+    oracle."""
+    w = W.CONFIGS["mimic"]
+    tr = cg.generate(w.gen, 3_000, 2_500)
+    t16, oor = cg.pack16(tr)
+    assert int(oor.item()) == 0
+    summ = np.zeros((1, 2_500), cg.SUMMARY_DTYPE)
+    st = cg.replay_host16(t16.pin(), w.cap, (policy,), trace_id_base=3_000, rand_seed=w.rand_seed,
+                          ovh=w.ovh, chunk=700, summary=summ)
+    ref = orc.replay_range(w, policy, 3_000, 5_500)
+    for f in SUMMARY_FIELDS:
+        np.testing.assert_array_equal(summ[0][f], ref[f].astype(summ[0][f].dtype), err_msg=f)
+    for k, v in ref["stats"].items():
+        assert cg.stats_dict(st[0])[k] == v, (policy, k)
+    b = W.random_batch(74, 600, 5, 1, 40, mode="valid", limit_choices=range(0, 41))
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
+    t16, oor = cg.pack16(tr)
+    summ = np.zeros((1, 600), cg.SUMMARY_DTYPE)
+    st = cg.replay_host16(t16.pin(), 40, (policy,), chunk=256, summary=summ)
+    ref = orc.replay_batch(b, 40, policy)
+    for f in SUMMARY_FIELDS:
+        np.testing.assert_array_equal(summ[0][f], ref[f].astype(summ[0][f].dtype), err_msg=f)
