@@ -250,8 +250,9 @@ int convgpu_replay_host(const convgpu_traces_t *host_traces, uint64_t n,
  *   op_delta[(i*n_ops + k)*n_containers + c]                   u16
  *   op_kinds[i*n_containers + c]                               u8: kind of op k in bits 2k, 2k+1
  * A trace is representable when every arrival, limit, op size and delta is
- * <= 0xFFFF (all BASELINE configs [0]-[4] are); convgpu_pack16 counts the
- * values that are not. */
+ * <= 0xFFFF (BASELINE configs [2]-[4] are; config [1] and the paper-mimic
+ * workload space containers 5,000 ticks apart, so their later arrivals are
+ * not); convgpu_pack16 counts the values that are not. */
 typedef struct {
   const uint16_t *arrival, *limit, *op_size, *op_delta; /* host (pinned for full speed) */
   const uint8_t *op_kinds;

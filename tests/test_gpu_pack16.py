@@ -117,10 +117,16 @@ def test_replay_host16_edge_batches(cg, orc, policy):
 
 @pytest.mark.parametrize("policy", ["fifo", "best_fit", "recent_fit", "random_fit"])
 def test_replay_host16_other_shapes(cg, orc, policy):
-    """The 16-bit host path with K = 2 (paper-mimic, n = 38, 66-MiB context)
-    and K = 1 (FINISH-only programs, n = 5): summaries and stats vs the
-    oracle."""
+    """The 16-bit host path with K = 2 (paper-mimic programs, n = 38, 66-MiB
+    context; arrivals 500 ticks apart so that they fit 16 bits — the paper's
+    5,000-tick spacing does not, and pack16 counts it) and K = 1
+    (FINISH-only programs, n = 5): summaries and stats vs the oracle."""
+    import dataclasses
     w = W.CONFIGS["mimic"]
+    tr = cg.generate(w.gen, 3_000, 100)
+    _, oor = cg.pack16(tr)
+    assert int(oor.item()) == 100 * 24  # arrivals 5,000 x c > 0xFFFF for c = 14 .. 37
+    w = dataclasses.replace(w, gen=dataclasses.replace(w.gen, iat=500))
     tr = cg.generate(w.gen, 3_000, 2_500)
     t16, oor = cg.pack16(tr)
     assert int(oor.item()) == 0
