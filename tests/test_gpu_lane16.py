@@ -349,3 +349,60 @@ def test_lane16_literal_mixed_fallback(cg, orc, policy):
     out = _gpu_replay(cg, tr, cap, policy + "+literal", seed=7, ovh=ovh, kernel="lane16")
     _compare(cg, out, ref)
     _compare_stats(cg, out, ref["stats"])
+
+
+def _boundary_batch(seed):
+    """Traces at the edges of the compact kernel's 16-bit fields and horizon:
+    limits 0xFFFE (fits) / 0xFFFF (does not), deltas 0xFFFF / 0x10000, op
+    sizes 0xFFFF / 0x10000 (above every 16-bit limit: rejected either way),
+    horizons 2^25 - 1 / 2^25 (compact) and 2^26 - 1 / 2^26 (TICK_RANGE), on a
+    capacity of 2^26 - 1 MiB.  Each trace's other values are small."""
+    rng = np.random.default_rng(seed)
+    n, K = 64, 4
+    base = W.random_batch(seed, 48, n, K, 200, ovh=3, mode="valid", limit_choices=range(4, 201))
+    arrival, limit = base.arrival.copy(), base.limit.copy()
+    delta, arg = base.delta.copy(), base.arg.copy()
+    cases = []
+    for i in range(48):
+        c = int(rng.integers(0, n))
+        kind = i % 8
+        if kind == 0:
+            limit[i, c] = 0xFFFE
+        elif kind == 1:
+            limit[i, c] = 0xFFFF
+        elif kind == 2:
+            delta[i, 1, c] = 0xFFFF
+        elif kind == 3:
+            delta[i, 1, c] = 0x10000
+        elif kind == 4:
+            arg[i, 0, c] = W.op(W.ALLOC, 0xFFFF)
+        elif kind == 5:
+            arg[i, 0, c] = W.op(W.ALLOC, 0x10000)
+        else:  # horizon = max arrival + sum of deltas
+            h = int(arrival[i].max()) + int(delta[i].astype(np.uint64).sum())
+            target = (1 << 25) - 1 if kind == 6 else (1 << 25)
+            if i % 16 >= 8:
+                target = (1 << 26) - 1 if kind == 6 else (1 << 26)
+            # the last container arrives late enough that the horizon hits the
+            # target exactly (arrivals stay sorted, every delta stays small)
+            arrival[i, n - 1] += np.uint32(target - h)
+        cases.append(kind)
+    return W.Batch(n, K, arrival, limit, delta, arg), cases
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_field_boundaries(cg, orc, policy):
+    """Every boundary of the compact layout against the oracle, element by
+    element: values that fit are replayed by the compact kernel, the others by
+    the marked fallback pass, and the TICK_RANGE traces are flagged, with the
+    same outputs either way."""
+    b, _ = _boundary_batch(404)
+    cap = (1 << 26) - 1
+    ref = orc.replay_batch(b, cap, policy, tid_base=77, rand_seed=5, ovh=3)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=77)
+    for kernel, full in (("lane16", True), ("lane16", False), ("lane", True), ("warp", True)):
+        out = _gpu_replay(cg, tr, cap, policy, seed=5, ovh=3, kernel=kernel, full=full)
+        _compare(cg, out, ref, full=full)
+        _compare_stats(cg, out, ref["stats"])
+    flags = ref["flags"]
+    assert (flags & (1 << 5)).any() and (flags == 0).sum() > 20  # TICK_RANGE present, most valid
