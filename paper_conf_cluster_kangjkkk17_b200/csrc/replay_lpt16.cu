@@ -72,7 +72,10 @@ constexpr uint32_t kNoC = 64u;
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kCompactHorizon = 1u << 25;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
-constexpr uint32_t kTmemCols = 128;
+// TMEM per warp: 64 columns of per-container sums + 32 of statistics
+// accumulators (20 used); warps w and w + 4 share a lane quarter
+constexpr uint32_t kTmemCols = 256;
+constexpr uint32_t kWarpCols = 128;
  // 64 per warp, warps w and w + 4 share a lane quarter
 
 // bytes per lane (= per trace) and warps per CTA (one CTA per SM)
@@ -147,25 +150,43 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // computed without re-reading the trace in the epilogue).  Computed in
   // registers by init, parked in this thread's TMEM lane for the whole event
   // loop (64 columns), read back for the epilogue: the loop does not carry 64
-  // registers for it.
+  // registers for it.  The thread's statistics accumulators (only touched by
+  // the epilogue) are parked the same way (20 more columns).
   uint32_t base[64];
   __shared__ uint32_t s_tmem;
   if (wib == 0) lpt::tmem_alloc(&s_tmem, kTmemCols);
   lpt::tmem_fence_before_sync();
   __syncthreads();
   lpt::tmem_fence_after_sync();
-  const uint32_t t_base = s_tmem + ((32u * (wib & 3u)) << 16) + (wib >> 2) * 64u;
-  auto park_base = [&]() {  // whole warp, converged
+  const uint32_t t_base = s_tmem + ((32u * (wib & 3u)) << 16) + (wib >> 2) * kWarpCols;
+  auto park_state = [&]() {  // whole warp, converged
     __syncwarp();
 #pragma unroll
     for (int q = 0; q < 4; ++q) lpt::tmem_st16(t_base + 16u * q, base + 16 * q);
+    uint32_t sr[32];
+    const unsigned long long u[9] = {st_traces, st_events, st_mk, st_wait, st_rej, st_sel, st_dig,
+                                     racc_r, racc};
+#pragma unroll
+    for (int j = 0; j < 9; ++j) { sr[2 * j] = (uint32_t)u[j]; sr[2 * j + 1] = (uint32_t)(u[j] >> 32); }
+    sr[18] = st_maxmk; sr[19] = st_maxpk;
+#pragma unroll
+    for (int j = 20; j < 32; ++j) sr[j] = 0;
+    lpt::tmem_st16(t_base + 64u, sr);
+    lpt::tmem_st16(t_base + 80u, sr + 16);
   };
-  auto fetch_base = [&]() {  // whole warp, converged
+  auto fetch_state = [&]() {  // whole warp, converged
     __syncwarp();
     lpt::tmem_wait_st();
 #pragma unroll
     for (int q = 0; q < 4; ++q) lpt::tmem_ld16(t_base + 16u * q, base + 16 * q);
+    uint32_t sr[32];
+    lpt::tmem_ld16(t_base + 64u, sr);
+    lpt::tmem_ld16(t_base + 80u, sr + 16);
     lpt::tmem_wait_ld();
+    auto u64 = [&](int j) { return (unsigned long long)sr[2 * j] | ((unsigned long long)sr[2 * j + 1] << 32); };
+    st_traces = u64(0); st_events = u64(1); st_mk = u64(2); st_wait = u64(3); st_rej = u64(4);
+    st_sel = u64(5); st_dig = u64(6); racc_r = u64(7); racc = u64(8);
+    st_maxmk = sr[18]; st_maxpk = sr[19];
   };
   uint32_t arr0 = 0;
   // Best-Fit (R3, R4): the trace's distinct limits in ascending order (unused
@@ -392,7 +413,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
   if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
-  park_base();
+  park_state();
   while (__any_sync(kFull, have)) {
     do {
       if (have && !tdone) {
@@ -623,15 +644,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         }
       }
     } while (!__all_sync(kFull, !have || tdone));
-    fetch_base();
+    fetch_state();
     if (have) {
       if (!skip) epilogue(i);
       i += T;
       have = i < p.count;
       if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
     }
-    park_base();
+    park_state();
   }
+  fetch_state();  // the statistics accumulators, for the final reduction
 #undef ASG
 #undef LIM
 #undef AT
