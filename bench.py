@@ -356,7 +356,9 @@ def run_ours(args, rank, local_rank, world):
     full = args.outputs == "full"
     outs = {p: cg.alloc_out(Nr, n, device=dev, full=full, stats=False) for p in POLICIES}
     nsteps = args.warmup + args.steps
-    stats = {p: torch.zeros(nsteps, 12, dtype=torch.int64, device=dev) for p in POLICIES}
+    # one [policies, 12] block of convgpu_stats_t records per step
+    stats_blk = torch.zeros(nsteps, len(POLICIES), 12, dtype=torch.int64, device=dev)
+    stats = {p: stats_blk[:, q] for q, p in enumerate(POLICIES)}
     ev_s = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
     ev_e = {p: [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)] for p in POLICIES}
     step_ev = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
@@ -371,8 +373,8 @@ def run_ours(args, rank, local_rank, world):
                       kernel=args.kernel)
             if timed_idx is not None:
                 ev_e[p][timed_idx].record(stream)
-            if world > 1:
-                cgd.reduce_stats(stats[p][s])
+        if world > 1:  # the step's exchange: every policy's record, two collectives
+            cgd.reduce_stats_block(stats_blk[s])
 
     for s in range(args.warmup):
         step(s)

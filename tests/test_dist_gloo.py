@@ -49,7 +49,10 @@ def _worker(rank, world, port, policy, q):
         lo, hi = cgd.shard_range(TOTAL, rank, world)
         r = oracle.replay_range(w, policy, lo, hi)
         st = _pack(r["stats"])
+        blk = torch.stack([st, st]).contiguous()  # the batched form: two records at once
         cgd.reduce_stats(st)
+        cgd.reduce_stats_block(blk)
+        assert (blk[0] == st).all() and (blk[1] == st).all()
         rdu = np.zeros((TOTAL + RANGE - 1) // RANGE, np.uint64)
         with np.errstate(over="ignore"):
             np.add.at(rdu, (lo + np.arange(hi - lo)) // RANGE, r["digest"].astype(np.uint64))
