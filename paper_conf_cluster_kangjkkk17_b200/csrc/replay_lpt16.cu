@@ -72,6 +72,11 @@ constexpr uint32_t kNoC = 64u;
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kCompactHorizon = 1u << 25;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
+#ifndef LPT16_SKIP
+#define LPT16_SKIP 0
+#endif
+// skip of admitted containers' passive ops (see the EVENT step)
+constexpr uint32_t kSkipped = 1u << 30;      // ust: ops after the skip left the event loop
 // TMEM per warp: 64 columns of per-container sums + 32 of statistics
 // accumulators (20 used); warps w and w + 4 share a lane quarter
 constexpr uint32_t kTmemCols = 256;
@@ -113,6 +118,7 @@ template <int POLICY>
 __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
   constexpr bool LIT = is_lit(POLICY);     // R1-LIT (NEXT-1) instead of R1
+  constexpr bool SKIP = LPT16_SKIP && !LIT;
   constexpr int P = POLICY & 0xFF;         // convgpu_policy_t
   const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
   constexpr uint32_t n = N, K = KOPS;
@@ -152,17 +158,17 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // loop (64 columns), read back for the epilogue: the loop does not carry 64
   // registers for it.  The thread's statistics accumulators (only touched by
   // the epilogue) are parked the same way (20 more columns).
-  uint32_t base[64];
   __shared__ uint32_t s_tmem;
   if (wib == 0) lpt::tmem_alloc(&s_tmem, kTmemCols);
   lpt::tmem_fence_before_sync();
   __syncthreads();
   lpt::tmem_fence_after_sync();
   const uint32_t t_base = s_tmem + ((32u * (wib & 3u)) << 16) + (wib >> 2) * kWarpCols;
+  // init parks the sums 16 containers at a time and the epilogue loads them
+  // the same way (both run converged, for every lane of the warp), so at
+  // most 16 of them are ever live in registers
   auto park_state = [&]() {  // whole warp, converged
     __syncwarp();
-#pragma unroll
-    for (int q = 0; q < 4; ++q) lpt::tmem_st16(t_base + 16u * q, base + 16 * q);
     uint32_t sr[32];
     const unsigned long long u[9] = {st_traces, st_events, st_mk, st_wait, st_rej, st_sel, st_dig,
                                      racc_r, racc};
@@ -177,8 +183,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   auto fetch_state = [&]() {  // whole warp, converged
     __syncwarp();
     lpt::tmem_wait_st();
-#pragma unroll
-    for (int q = 0; q < 4; ++q) lpt::tmem_ld16(t_base + 16u * q, base + 16 * q);
     uint32_t sr[32];
     lpt::tmem_ld16(t_base + 64u, sr);
     lpt::tmem_ld16(t_base + 80u, sr + 16);
@@ -205,8 +209,15 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // the op fetched in the previous iteration: container, op word, delta
   uint32_t pre_c = kNoC;
   bool skip = false;
+  // skip of an admitted container: the deltas of its FINISH tick are in
+  // flight (pre_skip); the tail stores the FINISH key when they land
+  bool pre_skip = false, skip_two = false;
+  uint32_t skip_acc = 0;
 #ifdef LPT16_DEBUG
   uint32_t dbg0 = 0, dbg1 = 0, dbg2 = 0, dbg3 = 0, dbg4 = 0;
+#endif
+#ifdef LPT16_COUNT  // experiment only: micro-step counters in the summary
+  uint32_t cnt_ev = 0, cnt_ds = 0, cnt_hz = 0, cnt_it = 0;
 #endif
   const uint32_t* trace_delta = nullptr;
   const uint32_t* trace_arg = nullptr;
@@ -223,7 +234,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     for (uint32_t j = 0; j < 8; ++j) gmin[j] = (j == g) ? m : gmin[j];
   };
 
-  auto init = [&](uint64_t ti) {
+  // Called by every lane of the warp (converged: it parks to TMEM); a lane
+  // without a trace (act = false) replays trace 0's loads with no global side
+  // effect and its state is never used.
+  auto init = [&](uint64_t ti, bool act) {
+    uint32_t base[16];
     const uint4* A4 = reinterpret_cast<const uint4*>(p.arrival + ti * n);
     const uint4* L4 = reinterpret_cast<const uint4*>(p.limit + ti * n);
     trace_delta = p.delta + ti * (uint64_t)K * n;
@@ -265,8 +280,12 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         LIM(c) = (uint16_t)min(L, 0xFFFFu);
         if (LIT) ASG(c) = 0;
         gmin[c >> 3] = min(gmin[c >> 3], key);
-        base[c] = bsum;
+        base[c & 15] = bsum;
         if (c == 0) arr0 = a;
+      }
+      if ((q & 3) == 3) {  // park 16 sums (R17's wait) in this thread's TMEM lane
+        __syncwarp();
+        lpt::tmem_st16(t_base + 4u * (q & ~3u), base);
       }
 
     }
@@ -276,7 +295,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     // container 0's slot doubles as the fallback mark; clear a stale mark a
     // previous call may have left in caller scratch (admissions of container
     // 0 are only read back when it was admitted, so 0 is harmless)
-    adm_out[0] = skip ? kLpt16Mark : 0u;
+    if (act) adm_out[0] = skip ? kLpt16Mark : 0u;
     if (P == CONVGPU_BEST_FIT && !LIT) {
       // distinct limits (unsorted while collected), with member masks
       uint32_t ncls = 0;
@@ -321,7 +340,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       // more distinct limits than classes: the 32-bit kernel replays it
       if (bad == 0 && ncls > (uint32_t)kBfClasses && !skip) {
         skip = true;
-        adm_out[0] = kLpt16Mark;
+        if (act) adm_out[0] = kLpt16Mark;
       }
     }
     flags = bad;
@@ -330,10 +349,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     pm_lo = pm_hi = 0;
     pre_c = kNoC;
     ru_head = kNoC;
+    pre_skip = false;
   };
 
-  auto epilogue = [&](uint64_t ti) {
+  // Called by every lane of the warp (converged: it loads from TMEM); only
+  // lanes with act = true store or count anything.
+  auto epilogue = [&](uint64_t ti, bool act) {
     lpt::cp_wait0();
+    uint32_t base[16];
     const bool stopped = (flags & kStopMask) != 0;
     if (stopped) { peak_res = 0; peak_used = 0; n_rej = 0; n_sel = 0; }
     uint64_t dig = 0, swait = 0;
@@ -342,6 +365,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
 #pragma unroll
     for (uint32_t q = 0; q < 16; ++q) {
+      if ((q & 3) == 0) {  // the next 16 parked sums
+        __syncwarp();
+        lpt::tmem_ld16(t_base + 4u * q, base);
+        lpt::tmem_wait_ld();
+      }
       // admissions this thread stored during the replay (coherent load)
       const uint4 m4 = stopped ? make_uint4(0, 0, 0, 0) : M4[q];
       uint32_t at[4], ar[4], wt[4], fn[4];
@@ -357,7 +385,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           }
           fn[j] = AT(s_key, c) & ~kDone;
           // R17: wait = finish - arrival - sum of deltas
-          wt[j] = fn[j] - base[c];
+          wt[j] = fn[j] - base[c & 15];
         }
         const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
         dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
@@ -366,19 +394,22 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       }
       // streaming stores (evict-first): outputs are not re-read, inputs of the
       // traces in flight should stay in L2
-      if (p.admit_tick)
+      if (act && p.admit_tick)
         __stcs(reinterpret_cast<uint4*>(p.admit_tick + ob) + q, make_uint4(at[0], at[1], at[2], at[3]));
-      if (p.admit_rank)
+      if (act && p.admit_rank)
         __stcs(reinterpret_cast<unsigned int*>(p.admit_rank + ob) + q,
                ar[0] | (ar[1] << 8) | (ar[2] << 16) | (ar[3] << 24));
-      if (p.wait) __stcs(reinterpret_cast<uint4*>(p.wait + ob) + q, make_uint4(wt[0], wt[1], wt[2], wt[3]));
-      if (p.finish) __stcs(reinterpret_cast<uint4*>(p.finish + ob) + q, make_uint4(fn[0], fn[1], fn[2], fn[3]));
+      if (act && p.wait)
+        __stcs(reinterpret_cast<uint4*>(p.wait + ob) + q, make_uint4(wt[0], wt[1], wt[2], wt[3]));
+      if (act && p.finish)
+        __stcs(reinterpret_cast<uint4*>(p.finish + ob) + q, make_uint4(fn[0], fn[1], fn[2], fn[3]));
     }
     const uint32_t makespan = stopped ? 0u : mfin - arr0;
     dig += mix64(((uint64_t)makespan << 32) | peak_res);
     dig += mix64(((uint64_t)peak_used << 32) | flags);
     dig += mix64(swait);
     dig += mix64(((uint64_t)n_rej << 32) | n_sel);
+    if (!act) return;
     if (p.summary) {
       convgpu_summary_t sm;
       sm.makespan = makespan; sm.peak_reserved = peak_res; sm.peak_used = peak_used;
@@ -389,6 +420,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         sm.makespan = dbg0; sm.peak_reserved = dbg1; sm.peak_used = dbg2; sm.n_rejected = dbg3;
         sm.n_select = dbg4; sm.sum_wait = events;
       }
+#endif
+#ifdef LPT16_COUNT
+      sm.makespan = cnt_ev; sm.peak_reserved = cnt_ds; sm.peak_used = cnt_hz; sm.n_rejected = cnt_it;
+      cnt_ev = cnt_ds = cnt_hz = cnt_it = 0;
 #endif
       p.summary[ti] = sm;
     }
@@ -412,12 +447,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
 
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
-  if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
+  if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; }
   park_state();
   while (__any_sync(kFull, have)) {
     do {
       if (have && !tdone) {
         uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
+        bool sk_now = false;             // this step skips a container (SKIP)
+        uint32_t sk_acc = 0;
         // next event (a2).  If it belongs to the container whose next op was
         // fetched in the previous iteration (rare), this lane idles for one
         // iteration: the tail below retires that fetch into the container's
@@ -426,6 +463,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         const uint32_t m45 = min(gmin[4], gmin[5]), m67 = min(gmin[6], gmin[7]);
         const uint32_t kmin = min(min(m01, m23), min(m45, m67));
         const bool hz = (kmin & 63u) == pre_c && kmin < kDone;
+#ifdef LPT16_COUNT
+        cnt_it++; cnt_ev += (!dmode && !hz) ? 1u : 0u; cnt_ds += dmode ? 1u : 0u; cnt_hz += (!dmode && hz) ? 1u : 0u;
+#endif
         if (!dmode && !hz) {
           // ================= EVENT step (a2 + a3), branch-free =================
           if (kmin >= kDone) {
@@ -434,9 +474,14 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           } else {
             const uint32_t t = kmin >> 6, c = kmin & 63u;
             cur_t = t;
-            ++events;
             const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
-            const bool arr = (ust & kNotArrived) == kNotArrived;
+            // SKIP: a skipped container's key was raised to its FINISH key
+            // after the group minimum took the key of its next op (a lower
+            // bound); such a stale minimum only re-mins its group
+            const uint32_t kcur = SKIP ? AT(s_key, c) : kmin;
+            const bool stale = SKIP && kcur != kmin;
+            events += stale ? 0u : 1u;
+            const bool arr = !stale && (ust & kNotArrived) == kNotArrived;
             // ARRIVE (Fig. 3b/3c; R2)
             // R1-LIT: every newcomer takes what is free (no fill target)
             const uint32_t g = (arr && (LIT || target == kNoC)) ? min(L, free_mem) : 0u;
@@ -451,7 +496,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             // intermediate sample: the ARRIVE changes no used memory, and
             // cap - free only falls after it.
             const bool fz = arr && (ust & kUsedMask) == 0u;
-            const bool op = !arr || fz;
+            const bool op = !stale && (!arr || fz);
             events += fz ? 1u : 0u;
             const uint32_t ust1 = arr ? ((vadm ? kAdmitted : 0u) | (ust & kKindsMask)) : ust;
             const uint32_t tg1 = vtgt ? c : target;
@@ -511,10 +556,28 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             nu = isX ? (ust1 & ~kUsedMask) : nu;
             nu = pause ? (ust1 | kPaused) : nu;
             nu = (adv && op) ? nu + kKOne : nu;
-            AT(s_ust, c) = nu;
             kc = badfree ? kNoC : c;
             nkc = adv ? (((t + nd) << 6) | c) : (isX ? (kDone | t) : (kPausedKey | plink));
             pfk = (adv && op) ? k + 1u : 0xFFu;
+            if (SKIP) {
+              // An admitted container (a = L) never pauses again, and its
+              // ALLOC / FREE / NOP change nothing but its own used memory: its
+              // ops up to FINISH leave the event loop.  Its key keeps the next
+              // op's tick (a lower bound) while the remaining deltas are
+              // fetched; the tail raises it to the FINISH key next iteration.
+              // Not taken when the next op runs at this tick (its key could
+              // sort below keys already processed).
+              const uint32_t nk = k + 1u;
+              const bool skp = adv && op && (nu & kAdmitted) && nk + 2u <= K && nd != 0u;
+              nu = skp ? ((nu & ~(7u << kKShift)) | ((K - 1u) << kKShift) | kSkipped) : nu;
+              sts_if(&AT(s_sd, c), (t + nd) | (nk << 25), skp);
+              sk_acc = t + nd;
+              pfk = skp ? nk + 1u : pfk;
+              sk_now = skp;
+              events += skp ? K - 1u - nk : 0u;
+            }
+            nkc = stale ? kcur : nkc;
+            AT(s_ust, c) = nu;
           }
         } else if (dmode) {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
@@ -603,6 +666,20 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             if (used_total > cap - free_mem) flags |= CONVGPU_FLAG_OVERCOMMIT;
             uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
             nu |= full ? kAdmitted : 0u;
+            nkc = ((t + (sdt >> 16)) << 6) | tg;
+            pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
+            if (SKIP) {
+              // resumed and admitted by this fill: skip as in the EVENT step (a
+              // target admitted while running skips at its pending op's event)
+              const uint32_t nk = (nu >> kKShift) & 7u, ndd = sdt >> 16;
+              const bool skp = res && full && nk + 2u <= K && ndd != 0u;
+              nu = skp ? ((nu & ~(7u << kKShift)) | ((K - 1u) << kKShift) | kSkipped) : nu;
+              sts_if(&AT(s_sd, tg), (t + ndd) | (nk << 25), skp);
+              sk_acc = t + ndd;
+              pfk = skp ? nk + 1u : pfk;
+              sk_now = skp;
+              events += skp ? K - 1u - nk : 0u;
+            }
             AT(s_ust, tg) = nu;
             const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;
             pm_lo &= ~(shl_c(1u, tg) & rmask);
@@ -621,8 +698,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
               dmode = full && (pm_lo | pm_hi) != 0u;
             }
             kc = res ? tg : kNoC;
-            nkc = ((t + (sdt >> 16)) << 6) | tg;
-            pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
           }
         }
         // ---- shared tail: key update, group re-min, retire the previous
@@ -633,24 +708,41 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           regroup(kcs);
           // retire last iteration's fetch (issued one iteration ago)
           lpt::cp_wait0();  // nothing pending if nothing was fetched: no branch needed
-          sts_if(&AT(s_sd, pre_c & 63u), pack_sd(AT(s_stg, 0), AT(s_stg, 1)), pre_c != kNoC);
-          // op k word and the delta of op k+1 (clamped: FINISH never reads it)
+          const uint32_t w0 = AT(s_stg, 0), w1 = AT(s_stg, 1), pc = pre_c & 63u;
+          if (SKIP) {
+            // a skipped container's deltas landed: raise its key to the
+            // FINISH key (its group minimum may stay at the old key: see the
+            // stale test in the EVENT step); else pack the op into sd
+            const uint32_t kf = ((skip_acc + w0 + (skip_two ? w1 : 0u)) << 6) | pc;
+            sts_if(pre_skip ? &AT(s_key, pc) : &AT(s_sd, pc), pre_skip ? kf : pack_sd(w0, w1),
+                   pre_c != kNoC);
+          } else {
+            sts_if(&AT(s_sd, pc), pack_sd(w0, w1), pre_c != kNoC);
+          }
+          // op k word and the delta of op k+1 (clamped: FINISH never reads it);
+          // a skip fetches deltas k and k+1 instead (k = the first op after
+          // the skipped ones' first)
           const bool f = pfk < K;
           const uint32_t off = pfk * n + kcs;
-          lpt::cp_async4_if(&AT(s_stg, 0), trace_arg + off, f);
+          lpt::cp_async4_if(&AT(s_stg, 0), ((SKIP && sk_now) ? trace_delta : trace_arg) + off, f);
           lpt::cp_async4_if(&AT(s_stg, 1), trace_delta + min(pfk + 1u, K - 1u) * n + kcs, f);
           lpt::cp_commit();
           pre_c = f ? kcs : kNoC;
+          if (SKIP) {
+            pre_skip = sk_now;
+            skip_two = pfk + 1u < K;
+            skip_acc = sk_acc;
+          }
         }
       }
     } while (!__all_sync(kFull, !have || tdone));
     fetch_state();
+    epilogue(have ? i : 0, have && !skip);
     if (have) {
-      if (!skip) epilogue(i);
       i += T;
       have = i < p.count;
-      if (have) { init(i); tdone = flags != 0 || skip; dmode = false; }
     }
+    if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; dmode = false; }
     park_state();
   }
   fetch_state();  // the statistics accumulators, for the final reduction
