@@ -32,6 +32,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import re
 import os
 import statistics
 import subprocess
@@ -410,7 +411,7 @@ def run_ours(args, rank, local_rank, world):
         if Nr < sms * 40:
             return "warp"
         return "lane16" if (n == 64 and K == 4) else "lane"
-    launches_per_replay = {p: 2 if kernel_of(p) == "lane16" else 1 for p in POLICIES}
+    launches_per_replay = {p: 3 if kernel_of(p) == "lane16" else 1 for p in POLICIES}
     # correctness of the timed work: every timed launch replayed every trace
     last = args.warmup + args.steps - 1
     checks = {}
@@ -506,7 +507,8 @@ def run_ours(args, rank, local_rank, world):
     for p in POLICIES:
         pid = {"fifo": 0, "best_fit": 1, "recent_fit": 2, "random_fit": 3}[p]
         for kname, v in lim.items():
-            if kernel_of(p) == "lane16" and f"replay_lpt16_kernel<{pid}>" in kname:
+            # first-pass compact kernel: "<P>" (round 1) or "<P, 0>" (16-bit layout)
+            if kernel_of(p) == "lane16" and re.search(rf"replay_lpt16_kernel<{pid}(, (0|false))?>", kname):
                 ipe[p] = v
     if len(ipe) == len(POLICIES):
         inst = sum(ipe[p]["warp_instructions_per_event"] * Nr * per_trace_events for p in POLICIES)
@@ -776,7 +778,7 @@ def run_c3(args, rank, world, dev, cg, cgd):
                        "fields": ["range digest"] + ["totals: " + ",".join(RANGE_FIELDS[1:])],
                        "source": "tests/golden/c3_range_digests.json (C oracle, scripts/c3_oracle_digests.py)",
                        **({"mismatches": bad[:8]} if bad else {})},
-            "gpu_launches": args.steps * nchunks * (1 + 2 * len(POLICIES)),
+            "gpu_launches": args.steps * nchunks * (1 + 3 * len(POLICIES)),
             "clocks": clocks,
         }
         print(json.dumps(result), flush=True)

@@ -113,16 +113,26 @@ enum {
   CONVGPU_KERNEL_AUTO = 0,
   CONVGPU_KERNEL_WARP_PER_TRACE = 1, /* one warp per trace, TMA-staged trace */
   CONVGPU_KERNEL_LANE_PER_TRACE = 2, /* one lane per trace, 32 traces per warp */
-  CONVGPU_KERNEL_LANE_COMPACT = 3    /* one lane per trace, 16-bit packed state, up to
+  CONVGPU_KERNEL_LANE_COMPACT = 3,   /* one lane per trace, 16-bit packed state, up to
                                         8 warps per SM; needs n_containers = 64, n_ops = 4,
                                         out->admit_tick or out->admit_scratch != NULL (it
                                         holds admissions during the replay) and 16-byte
                                         aligned arrays / outputs,
                                         else -EINVAL.  Traces whose limits exceed 0xFFFE
-                                        MiB, deltas 0xFFFF ticks or horizon 2^25 are
-                                        replayed by a second, 32-bit lane-per-trace launch.
+                                        MiB are replayed by a second launch of the same
+                                        kernel with 17-bit limits / used memory (R1; if
+                                        every ALLOC / FREE size is <= 0xFFFE and every
+                                        limit <= 0x1FFFF), the rest, and traces whose
+                                        deltas exceed 0xFFFF ticks or horizon 2^25, by a
+                                        32-bit lane-per-trace launch (R1-LIT: the
+                                        warp-per-trace kernel).
                                         AUTO picks it whenever the lane kernel would run
                                         and these conditions hold. */
+  CONVGPU_KERNEL_LANE_COMPACT_WIDE = 4 /* the same with the 17-bit layout as the first
+                                        pass (R1; R1-LIT: as LANE_COMPACT): for batches
+                                        whose limits exceed 0xFFFE MiB (config [4] at
+                                        rho = 8), which would all take the second pass;
+                                        same requirements, same results */
 };
 
 /* Per-trace summary, 40 bytes. */
@@ -342,7 +352,8 @@ int convgpu_wrap_ops(const convgpu_api_op_t *api, uint64_t n, uint32_t n_contain
                      uint32_t n_ops, uint32_t pitch_align, uint32_t *op_arg, void *stream);
 
 /* Upper bound on the kernel launches convgpu_replay enqueues per call (the
- * compact lane kernel is followed by its 32-bit fallback pass; every other
+ * compact lane kernel is followed by its 17-bit and 32-bit fallback passes,
+ * which replay only the traces the previous pass marked; every other
  * variant launches once; convgpu_generate launches once;
  * convgpu_replay_host: this many per chunk and policy). */
 int convgpu_launches_per_call(void);

@@ -28,7 +28,7 @@ LITERAL = 0x100  # CONVGPU_DISPATCH_LITERAL: OR into a policy for the R1-LIT rea
 POLICY = {"fifo": FIFO, "best_fit": BEST_FIT, "recent_fit": RECENT_FIT, "random_fit": RANDOM_FIT}
 ALLOC, FREE, FINISH, NOP = 0, 1, 2, 3
 NONE32, NONE8 = 0xFFFFFFFF, 0xFF
-KERNEL = {"auto": 0, "warp": 1, "lane": 2, "lane16": 3}
+KERNEL = {"auto": 0, "warp": 1, "lane": 2, "lane16": 3, "lane16w": 4}
 FLAG_NAMES = ("deadlock", "overcommit", "invalid_limit", "invalid_free", "unsorted_arrival",
               "tick_range", "bad_program")
 
@@ -304,7 +304,9 @@ def replay(traces: Traces, capacity: int, policy, out: ReplayOut, rand_seed: int
     """Replay every trace of `traces` under `policy` (convgpu_replay).  Outputs
     go to the tensors of `out`; out.stats is accumulated (zero it first).
     kernel: "auto" | "warp" (warp per trace) | "lane" (lane per trace) |
-    "lane16" (lane per trace, compact state; n = 64, K = 4, admit_tick needed)."""
+    "lane16" (lane per trace, compact state; n = 64, K = 4, admit_tick or
+    admit_scratch needed) | "lane16w" (the same, 17-bit layout first: for
+    limits above 0xFFFE MiB)."""
     tr = traces.struct(rand_seed, ovh, kernel)
     o = OutT(_ptr(out.admit_tick), _ptr(out.admit_rank), _ptr(out.wait), _ptr(out.finish),
              _ptr(out.summary), _ptr(out.stats), _ptr(out.range_digest), out.range_size,

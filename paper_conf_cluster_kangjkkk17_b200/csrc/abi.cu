@@ -58,7 +58,7 @@ int validate_shape(const convgpu_traces_t* t, uint32_t cap, int policy) {
     return -EINVAL;
   if (cap == 0 || cap >= CONVGPU_CAPACITY_LIMIT) return -EINVAL;
   if (t->ctx_overhead_mib >= CONVGPU_OVERHEAD_LIMIT) return -EINVAL;
-  if (t->kernel_variant > CONVGPU_KERNEL_LANE_COMPACT) return -EINVAL;
+  if (t->kernel_variant > CONVGPU_KERNEL_LANE_COMPACT_WIDE) return -EINVAL;
   return 0;
 }
 
@@ -109,9 +109,9 @@ cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cuda
   // R1-LIT runs on the compact kernel or the warp-per-trace kernel
   if ((policy & CONVGPU_DISPATCH_LITERAL) && variant == CONVGPU_KERNEL_LANE_PER_TRACE)
     variant = CONVGPU_KERNEL_WARP_PER_TRACE;
-  if (variant == CONVGPU_KERNEL_LANE_COMPACT) {
+  if (variant == CONVGPU_KERNEL_LANE_COMPACT || variant == CONVGPU_KERNEL_LANE_COMPACT_WIDE) {
     if (!convgpu::lpt16_supported(a)) return cudaErrorInvalidValue;  // -EINVAL, see convgpu_replay
-    return convgpu::launch_replay_lpt16(a, policy, s);
+    return convgpu::launch_replay_lpt16(a, policy, s, variant == CONVGPU_KERNEL_LANE_COMPACT_WIDE);
   }
   if (variant == CONVGPU_KERNEL_LANE_PER_TRACE) return convgpu::launch_replay_lpt(a, policy, s);
   return convgpu::launch_replay(a, policy, use_bulk(a), s);
@@ -123,7 +123,7 @@ extern "C" {
 
 int convgpu_abi_version(void) { return CONVGPU_ABI_VERSION; }
 
-int convgpu_launches_per_call(void) { return 2; }  // compact lane kernel + its 32-bit fallback pass
+int convgpu_launches_per_call(void) { return 3; }  // compact lane kernel + its 17-bit and 32-bit fallback passes
 
 const char* convgpu_strerror(int rc) {
   switch (rc) {
@@ -141,7 +141,8 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   if (rc) return rc;
   if (!out) return -EINVAL;
   if (out->range_digest && out->range_size == 0) return -EINVAL;
-  if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT &&
+  if ((traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT ||
+       traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT_WIDE) &&
       (traces->n_containers != 64 || traces->n_ops != 4 || (!out->admit_tick && !out->admit_scratch)))
     return -EINVAL;
   if (n == 0) return 0;  // no-op: array pointers may be NULL
@@ -161,7 +162,8 @@ int convgpu_replay(const convgpu_traces_t* traces, uint64_t n, uint32_t capacity
   a.summary = out->summary; a.stats = out->stats;
   a.range_digest = out->range_digest; a.range_size = out->range_size;
   a.adm_scratch = out->admit_scratch;
-  if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT) {
+  if (traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT ||
+      traces->kernel_variant == CONVGPU_KERNEL_LANE_COMPACT_WIDE) {
     a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.adm_scratch) &&
                   aligned16(a.wait) && aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
     if (!convgpu::lpt16_supported(a)) return -EINVAL;

@@ -27,20 +27,25 @@ struct ReplayArgs {
   uint64_t grid_override;  // 0 = occupancy-sized persistent grid
   uint32_t per_sm_cap;     // tuning knob (env CONVGPU_PER_SM_CAP): at most this many CTAs per SM
   uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
-  uint32_t only_marked;    // lane kernel: replay only traces with adm_buf()[i*n] == kLpt16Mark
+  uint32_t only_marked;    // 0, or a mark: replay only traces with adm_buf()[i*n] == only_marked
   uint32_t* adm_scratch;   // compact kernel: admissions during the replay when admit_tick == NULL
 
   // where the compact kernel keeps admissions (and its fallback marks)
   __host__ __device__ uint32_t* adm_buf() const { return admit_tick ? admit_tick : adm_scratch; }
 };
 
-// admit_tick[i*n] of a trace the compact kernel left to the 32-bit lane kernel
+// admit_tick[i*n] (container 0's admission slot, above every admission
+// value) of a trace the compact kernel left to the next pass: the 16-bit
+// layout's to the 17-bit one (R1-LIT: to the warp-per-trace kernel), the
+// 17-bit layout's to the 32-bit lane kernel
 constexpr uint32_t kLpt16Mark = 0xFFFFFFFEu;
+constexpr uint32_t kLpt16Mark2 = 0xFFFFFFFDu;
 
 cudaError_t launch_replay(const ReplayArgs& a, int policy, bool bulk, cudaStream_t stream);
 cudaError_t launch_replay_lpt(const ReplayArgs& a, int policy, cudaStream_t stream);
 bool lpt16_supported(const ReplayArgs& a);
-cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream);
+cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream,
+                                bool wide_first = false);
 
 struct GenArgs {
   convgpu_gen_params_t p;

@@ -206,7 +206,7 @@ __global__ void __launch_bounds__(kReplayThreads, 8) replay_kernel(const ReplayA
       phase ^= 1u << b;
     } else {
       // fallback pass of the compact kernel (R1-LIT): only the traces it marked
-      if (p.only_marked && p.adm_buf()[i * n] != kLpt16Mark) continue;
+      if (p.only_marked && p.adm_buf()[i * n] != p.only_marked) continue;
       __syncwarp();
       prefetch(i, 0);
       __syncwarp();

@@ -377,7 +377,7 @@ __global__ void __launch_bounds__(kLptThreads) replay_lpt_kernel(const ReplayArg
       }
 #pragma unroll
       for (int u = 0; u < 8; ++u)
-        if (m[u] == kLpt16Mark) return j + (uint64_t)u * T;
+        if (m[u] == p.only_marked) return j + (uint64_t)u * T;
       j += 8 * T;
     }
     return j;

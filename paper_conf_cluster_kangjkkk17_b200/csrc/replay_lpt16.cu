@@ -55,16 +55,20 @@ using lpt::shl_c;
 using lpt::sts_if;
 
 constexpr uint32_t N = 64, KOPS = 4;  // compile-time shape (configs [2]-[4])
-// ust word
-constexpr uint32_t kUsedMask = 0xFFFFu;
-constexpr uint32_t kKShift = 16;
-constexpr uint32_t kKOne = 1u << kKShift;
-constexpr uint32_t kFirst = 1u << 19;
-constexpr uint32_t kPaused = 1u << 20;
-constexpr uint32_t kAdmitted = 1u << 21;
-constexpr uint32_t kNotArrived = kPaused | kAdmitted;
-constexpr uint32_t kKindShift = 22;
-constexpr uint32_t kKindsMask = 0xFFu << kKindShift;
+// ust word: used (16 bits; WIDE: 17) | op index 3 | FIRST | PAUSED | ADMITTED |
+// op kinds 2 x K (| WIDE: bit 16 of the declared limit, whose bits 0-15 are
+// in the u16 limit array)
+template <bool WIDE>
+struct Lay {
+  static constexpr uint32_t kUsedBits = WIDE ? 17u : 16u;
+  static constexpr uint32_t kUsedMask = (1u << kUsedBits) - 1u;
+  static constexpr uint32_t kKShift = kUsedBits;
+  static constexpr uint32_t kFirst = 1u << (kUsedBits + 3);
+  static constexpr uint32_t kPaused = 1u << (kUsedBits + 4);
+  static constexpr uint32_t kAdmitted = 1u << (kUsedBits + 5);
+  static constexpr uint32_t kKindShift = kUsedBits + 6;
+  static constexpr uint32_t kLimHi = WIDE ? 1u << 31 : 0u;
+};
 // keys
 constexpr uint32_t kDone = 0x80000000u;    // | finish tick
 constexpr uint32_t kPausedKey = 0xC0000000u;  // | suspension number
@@ -72,11 +76,6 @@ constexpr uint32_t kNoC = 64u;
 constexpr uint32_t kTickLimit = CONVGPU_TICK_LIMIT;
 constexpr uint32_t kCompactHorizon = 1u << 25;
 constexpr uint32_t kStopMask = ~(uint32_t)CONVGPU_FLAG_OVERCOMMIT;
-#ifndef LPT16_SKIP
-#define LPT16_SKIP 0
-#endif
-// skip of admitted containers' passive ops (see the EVENT step)
-constexpr uint32_t kSkipped = 1u << 30;      // ust: ops after the skip left the event loop
 // TMEM per warp: 64 columns of per-container sums + 32 of statistics
 // accumulators (20 used); warps w and w + 4 share a lane quarter
 constexpr uint32_t kTmemCols = 256;
@@ -114,11 +113,21 @@ __device__ __forceinline__ uint32_t pack_sd(uint32_t cw, uint32_t d) {
   return min(cw & kSizeMask, 0xFFFFu) | (d << 16);
 }
 
-template <int POLICY>
+// WIDE: the second pass over the traces the 16-bit layout could not hold
+// (marked kLpt16Mark by the first): 17-bit limits and used memory; traces it
+// cannot hold either are re-marked kLpt16Mark2 for the 32-bit kernel.
+template <int POLICY, bool WIDE>
 __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_kernel(const ReplayArgs p) {
   extern __shared__ __align__(16) uint32_t smem_w[];
+  using Ly = Lay<WIDE>;
+  constexpr uint32_t kUsedMask = Ly::kUsedMask, kKShift = Ly::kKShift, kKOne = 1u << kKShift;
+  constexpr uint32_t kFirst = Ly::kFirst, kPaused = Ly::kPaused, kAdmitted = Ly::kAdmitted;
+  constexpr uint32_t kNotArrived = kPaused | kAdmitted;
+  constexpr uint32_t kKindShift = Ly::kKindShift, kKindsMask = 0xFFu << kKindShift;
+  constexpr uint32_t kLimHi = Ly::kLimHi;
+  // the declared limit of a container whose ust word is u
+#define FULL_L(c, u) (WIDE ? (uint32_t)LIM(c) | (((u) >> 31) << 16) : (uint32_t)LIM(c))
   constexpr bool LIT = is_lit(POLICY);     // R1-LIT (NEXT-1) instead of R1
-  constexpr bool SKIP = LPT16_SKIP && !LIT;
   constexpr int P = POLICY & 0xFF;         // convgpu_policy_t
   const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
   constexpr uint32_t n = N, K = KOPS;
@@ -144,7 +153,25 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // run SM-first (slot = wib * gridDim + block), so the last, partial round
   // spreads over every SM instead of filling the first CTAs.
   const uint64_t T = (uint64_t)gridDim.x * blockDim.x;
-  uint64_t i = ((uint64_t)wib * gridDim.x + blockIdx.x) * 32u + lane;
+  // only_marked (the WIDE pass): the next trace from j on whose container-0
+  // admission slot holds the mark (8 markers probed per step, all in flight)
+  auto next = [&](uint64_t j) -> uint64_t {
+    if (!WIDE || !p.only_marked) return j;
+    while (j < p.count) {
+      uint32_t m[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint64_t jj = j + (uint64_t)u * T;
+        m[u] = jj < p.count ? p.adm_buf()[jj * N] : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (m[u] == p.only_marked) return j + (uint64_t)u * T;
+      j += 8 * T;
+    }
+    return j;
+  };
+  uint64_t i = next(((uint64_t)wib * gridDim.x + blockIdx.x) * 32u + lane);
 
   unsigned long long st_traces = 0, st_events = 0, st_mk = 0, st_wait = 0, st_rej = 0,
                      st_sel = 0, st_dig = 0;
@@ -209,10 +236,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   // the op fetched in the previous iteration: container, op word, delta
   uint32_t pre_c = kNoC;
   bool skip = false;
-  // skip of an admitted container: the deltas of its FINISH tick are in
-  // flight (pre_skip); the tail stores the FINISH key when they land
-  bool pre_skip = false, skip_two = false;
-  uint32_t skip_acc = 0;
 #ifdef LPT16_DEBUG
   uint32_t dbg0 = 0, dbg1 = 0, dbg2 = 0, dbg3 = 0, dbg4 = 0;
 #endif
@@ -246,7 +269,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     adm_out = p.adm_buf() + ti * n;
     const uint4* D4 = reinterpret_cast<const uint4*>(trace_delta);
     const uint4* R4 = reinterpret_cast<const uint4*>(trace_arg);
-    uint32_t bad = 0, lsum = 0, amax = 0, prev = 0, lmax = 0, dmax = 0;
+    uint32_t bad = 0, lsum = 0, amax = 0, prev = 0, lmax = 0, dmax = 0, smax = 0;
 #pragma unroll
     for (int j = 0; j < 8; ++j) gmin[j] = kKeyNone;
 #pragma unroll
@@ -271,13 +294,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           lsum = min(lsum + min(d, kTickLimit), kTickLimit);
           dmax = max(dmax, d);
           if (((w >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+          if (WIDE && ((w >> 30) == CONVGPU_OP_ALLOC || (w >> 30) == CONVGPU_OP_FREE))
+            smax = max(smax, w & kSizeMask);
           kinds |= (w >> 30) << (2 * k);
         }
         const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
         AT(s_key, c) = key;
-        AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu);
+        AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu) |
+                       (WIDE ? ((L >> 16) & 1u) << 31 : 0u);
         AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
-        LIM(c) = (uint16_t)min(L, 0xFFFFu);
+        LIM(c) = (uint16_t)(WIDE ? L : min(L, 0xFFFFu));  // WIDE: bit 16 in the ust word
         if (LIT) ASG(c) = 0;
         gmin[c >> 3] = min(gmin[c >> 3], key);
         base[c & 15] = bsum;
@@ -291,11 +317,16 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     }
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     // not representable in the 16-bit fields: the 32-bit kernel replays it
-    skip = bad == 0 && (lmax > 0xFFFEu || dmax > 0xFFFFu || amax + lsum >= kCompactHorizon);
+    // Op sizes are saturated at 0xFFFF, which is exact while every limit is
+    // <= 0xFFFE (a saturated size is above every limit, so rejected or
+    // flagged as the full size would be).  WIDE: limits and used memory have
+    // 17 bits and the sizes must fit exactly.
+    const bool lim_ok = WIDE ? (lmax <= 0x1FFFFu && smax <= 0xFFFEu) : lmax <= 0xFFFEu;
+    skip = bad == 0 && (!lim_ok || dmax > 0xFFFFu || amax + lsum >= kCompactHorizon);
     // container 0's slot doubles as the fallback mark; clear a stale mark a
     // previous call may have left in caller scratch (admissions of container
     // 0 are only read back when it was admitted, so 0 is harmless)
-    if (act) adm_out[0] = skip ? kLpt16Mark : 0u;
+    if (act) adm_out[0] = skip ? (WIDE ? kLpt16Mark2 : kLpt16Mark) : 0u;
     if (P == CONVGPU_BEST_FIT && !LIT) {
       // distinct limits (unsorted while collected), with member masks
       uint32_t ncls = 0;
@@ -303,7 +334,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       for (int j = 0; j < kBfClasses; ++j) { bl[j] = 0xFFFFFFFFu; bm_lo[j] = 0; bm_hi[j] = 0; }
 #pragma unroll
       for (int c = 0; c < 64; ++c) {
-        const uint32_t Lc = LIM(c), bit = 1u << (c & 31);
+        const uint32_t Lc = FULL_L(c, AT(s_ust, c)), bit = 1u << (c & 31);
         bool hit = false;
 #pragma unroll
         for (int j = 0; j < kBfClasses; ++j) {
@@ -340,7 +371,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       // more distinct limits than classes: the 32-bit kernel replays it
       if (bad == 0 && ncls > (uint32_t)kBfClasses && !skip) {
         skip = true;
-        if (act) adm_out[0] = kLpt16Mark;
+        if (act) adm_out[0] = WIDE ? kLpt16Mark2 : kLpt16Mark;
       }
     }
     flags = bad;
@@ -349,7 +380,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     pm_lo = pm_hi = 0;
     pre_c = kNoC;
     ru_head = kNoC;
-    pre_skip = false;
   };
 
   // Called by every lane of the warp (converged: it loads from TMEM); only
@@ -453,8 +483,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     do {
       if (have && !tdone) {
         uint32_t kc = kNoC, nkc = kKeyNone, pfk = 0xFFu;
-        bool sk_now = false;             // this step skips a container (SKIP)
-        uint32_t sk_acc = 0;
         // next event (a2).  If it belongs to the container whose next op was
         // fetched in the previous iteration (rare), this lane idles for one
         // iteration: the tail below retires that fetch into the container's
@@ -474,14 +502,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           } else {
             const uint32_t t = kmin >> 6, c = kmin & 63u;
             cur_t = t;
-            const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = LIM(c);
-            // SKIP: a skipped container's key was raised to its FINISH key
-            // after the group minimum took the key of its next op (a lower
-            // bound); such a stale minimum only re-mins its group
-            const uint32_t kcur = SKIP ? AT(s_key, c) : kmin;
-            const bool stale = SKIP && kcur != kmin;
-            events += stale ? 0u : 1u;
-            const bool arr = !stale && (ust & kNotArrived) == kNotArrived;
+            ++events;
+            const uint32_t ust = AT(s_ust, c), sd = AT(s_sd, c), L = FULL_L(c, ust);
+            const bool arr = (ust & kNotArrived) == kNotArrived;
             // ARRIVE (Fig. 3b/3c; R2)
             // R1-LIT: every newcomer takes what is free (no fill target)
             const uint32_t g = (arr && (LIT || target == kNoC)) ? min(L, free_mem) : 0u;
@@ -496,9 +519,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             // intermediate sample: the ARRIVE changes no used memory, and
             // cap - free only falls after it.
             const bool fz = arr && (ust & kUsedMask) == 0u;
-            const bool op = !stale && (!arr || fz);
+            const bool op = !arr || fz;
             events += fz ? 1u : 0u;
-            const uint32_t ust1 = arr ? ((vadm ? kAdmitted : 0u) | (ust & kKindsMask)) : ust;
+            const uint32_t ust1 = arr ? ((vadm ? kAdmitted : 0u) | (ust & (kKindsMask | kLimHi))) : ust;
             const uint32_t tg1 = vtgt ? c : target;
             const uint32_t k = (ust1 >> kKShift) & 7u;
             const uint32_t kind = (ust1 >> (kKindShift + 2 * k)) & 3u;
@@ -559,24 +582,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             kc = badfree ? kNoC : c;
             nkc = adv ? (((t + nd) << 6) | c) : (isX ? (kDone | t) : (kPausedKey | plink));
             pfk = (adv && op) ? k + 1u : 0xFFu;
-            if (SKIP) {
-              // An admitted container (a = L) never pauses again, and its
-              // ALLOC / FREE / NOP change nothing but its own used memory: its
-              // ops up to FINISH leave the event loop.  Its key keeps the next
-              // op's tick (a lower bound) while the remaining deltas are
-              // fetched; the tail raises it to the FINISH key next iteration.
-              // Not taken when the next op runs at this tick (its key could
-              // sort below keys already processed).
-              const uint32_t nk = k + 1u;
-              const bool skp = adv && op && (nu & kAdmitted) && nk + 2u <= K && nd != 0u;
-              nu = skp ? ((nu & ~(7u << kKShift)) | ((K - 1u) << kKShift) | kSkipped) : nu;
-              sts_if(&AT(s_sd, c), (t + nd) | (nk << 25), skp);
-              sk_acc = t + nd;
-              pfk = skp ? nk + 1u : pfk;
-              sk_now = skp;
-              events += skp ? K - 1u - nk : 0u;
-            }
-            nkc = stale ? kcur : nkc;
             AT(s_ust, c) = nu;
           }
         } else if (dmode) {
@@ -652,7 +657,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             // step follows a pause / FINISH (no fetch) or an admission, after
             // which the resumed container is no longer paused
             const uint32_t tg = target;
-            const uint32_t Lt = LIM(tg), ut = AT(s_ust, tg), sdt = AT(s_sd, tg);
+            const uint32_t ut = AT(s_ust, tg), sdt = AT(s_sd, tg), Lt = FULL_L(tg, ut);
             const uint32_t g = min(free_mem, Lt - a_tg);
             a_tg += g;
             free_mem -= g;
@@ -668,18 +673,6 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             nu |= full ? kAdmitted : 0u;
             nkc = ((t + (sdt >> 16)) << 6) | tg;
             pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
-            if (SKIP) {
-              // resumed and admitted by this fill: skip as in the EVENT step (a
-              // target admitted while running skips at its pending op's event)
-              const uint32_t nk = (nu >> kKShift) & 7u, ndd = sdt >> 16;
-              const bool skp = res && full && nk + 2u <= K && ndd != 0u;
-              nu = skp ? ((nu & ~(7u << kKShift)) | ((K - 1u) << kKShift) | kSkipped) : nu;
-              sts_if(&AT(s_sd, tg), (t + ndd) | (nk << 25), skp);
-              sk_acc = t + ndd;
-              pfk = skp ? nk + 1u : pfk;
-              sk_now = skp;
-              events += skp ? K - 1u - nk : 0u;
-            }
             AT(s_ust, tg) = nu;
             const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;
             pm_lo &= ~(shl_c(1u, tg) & rmask);
@@ -708,44 +701,28 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
           regroup(kcs);
           // retire last iteration's fetch (issued one iteration ago)
           lpt::cp_wait0();  // nothing pending if nothing was fetched: no branch needed
-          const uint32_t w0 = AT(s_stg, 0), w1 = AT(s_stg, 1), pc = pre_c & 63u;
-          if (SKIP) {
-            // a skipped container's deltas landed: raise its key to the
-            // FINISH key (its group minimum may stay at the old key: see the
-            // stale test in the EVENT step); else pack the op into sd
-            const uint32_t kf = ((skip_acc + w0 + (skip_two ? w1 : 0u)) << 6) | pc;
-            sts_if(pre_skip ? &AT(s_key, pc) : &AT(s_sd, pc), pre_skip ? kf : pack_sd(w0, w1),
-                   pre_c != kNoC);
-          } else {
-            sts_if(&AT(s_sd, pc), pack_sd(w0, w1), pre_c != kNoC);
-          }
-          // op k word and the delta of op k+1 (clamped: FINISH never reads it);
-          // a skip fetches deltas k and k+1 instead (k = the first op after
-          // the skipped ones' first)
+          sts_if(&AT(s_sd, pre_c & 63u), pack_sd(AT(s_stg, 0), AT(s_stg, 1)), pre_c != kNoC);
+          // op k word and the delta of op k+1 (clamped: FINISH never reads it)
           const bool f = pfk < K;
           const uint32_t off = pfk * n + kcs;
-          lpt::cp_async4_if(&AT(s_stg, 0), ((SKIP && sk_now) ? trace_delta : trace_arg) + off, f);
+          lpt::cp_async4_if(&AT(s_stg, 0), trace_arg + off, f);
           lpt::cp_async4_if(&AT(s_stg, 1), trace_delta + min(pfk + 1u, K - 1u) * n + kcs, f);
           lpt::cp_commit();
           pre_c = f ? kcs : kNoC;
-          if (SKIP) {
-            pre_skip = sk_now;
-            skip_two = pfk + 1u < K;
-            skip_acc = sk_acc;
-          }
         }
       }
     } while (!__all_sync(kFull, !have || tdone));
     fetch_state();
     epilogue(have ? i : 0, have && !skip);
     if (have) {
-      i += T;
+      i = next(i + T);
       have = i < p.count;
     }
     if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; dmode = false; }
     park_state();
   }
   fetch_state();  // the statistics accumulators, for the final reduction
+#undef FULL_L
 #undef ASG
 #undef LIM
 #undef AT
@@ -785,9 +762,9 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
   if (wib == 0) lpt::tmem_dealloc(s_tmem, kTmemCols);
 }
 
-template <int POLICY>
+template <int POLICY, bool WIDE = false>
 static cudaError_t launch_t(const ReplayArgs& a, cudaStream_t stream) {
-  auto kern = replay_lpt16_kernel<POLICY>;
+  auto kern = replay_lpt16_kernel<POLICY, WIDE>;
   int dev = 0, sms = 0;
   cudaError_t e;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
@@ -819,10 +796,26 @@ bool lpt16_supported(const ReplayArgs& a) {
   return a.n == lpt16::N && a.K == lpt16::KOPS && a.adm_buf() != nullptr && a.aligned16;
 }
 
-cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream) {
+cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t stream,
+                                bool wide_first) {
   cudaError_t e;
   const bool lit = (policy & CONVGPU_DISPATCH_LITERAL) != 0;
   constexpr int L = CONVGPU_DISPATCH_LITERAL;
+  ReplayArgs b = a;
+  if (wide_first && !lit) {
+    // CONVGPU_KERNEL_LANE_COMPACT_WIDE: the 17-bit layout over every trace,
+    // what it cannot hold (kLpt16Mark2) to the 32-bit lane kernel
+    switch (policy & 0xFF) {
+      case CONVGPU_FIFO: e = lpt16::launch_t<CONVGPU_FIFO, true>(a, stream); break;
+      case CONVGPU_BEST_FIT: e = lpt16::launch_t<CONVGPU_BEST_FIT, true>(a, stream); break;
+      case CONVGPU_RECENT_FIT: e = lpt16::launch_t<CONVGPU_RECENT_FIT, true>(a, stream); break;
+      case CONVGPU_RANDOM_FIT: e = lpt16::launch_t<CONVGPU_RANDOM_FIT, true>(a, stream); break;
+      default: return cudaErrorInvalidValue;
+    }
+    if (e != cudaSuccess) return e;
+    b.only_marked = kLpt16Mark2;
+    return launch_replay_lpt(b, policy, stream);
+  }
   switch ((policy & 0xFF) | (lit ? L : 0)) {
     case CONVGPU_FIFO: e = lpt16::launch_t<CONVGPU_FIFO>(a, stream); break;
     case CONVGPU_BEST_FIT: e = lpt16::launch_t<CONVGPU_BEST_FIT>(a, stream); break;
@@ -835,11 +828,25 @@ cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t st
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  // traces the 16-bit layout cannot hold: the 32-bit lane kernel, marked only
-  // (R1-LIT: the warp-per-trace kernel, which implements that reading)
-  ReplayArgs b = a;
-  b.only_marked = 1;
-  return lit ? launch_replay(b, policy, false, stream) : launch_replay_lpt(b, policy, stream);
+  b.only_marked = kLpt16Mark;
+  // R1-LIT: the traces the 16-bit layout cannot hold go to the warp-per-trace
+  // kernel (which implements that reading), marked only
+  if (lit) return launch_replay(b, policy, false, stream);
+  // R1: to the 17-bit layout (WIDE), marked only; what that cannot hold
+  // either (re-marked kLpt16Mark2) to the 32-bit lane kernel
+#ifdef LPT16_NO_WIDE
+  return launch_replay_lpt(b, policy, stream);
+#endif
+  switch (policy & 0xFF) {
+    case CONVGPU_FIFO: e = lpt16::launch_t<CONVGPU_FIFO, true>(b, stream); break;
+    case CONVGPU_BEST_FIT: e = lpt16::launch_t<CONVGPU_BEST_FIT, true>(b, stream); break;
+    case CONVGPU_RECENT_FIT: e = lpt16::launch_t<CONVGPU_RECENT_FIT, true>(b, stream); break;
+    case CONVGPU_RANDOM_FIT: e = lpt16::launch_t<CONVGPU_RANDOM_FIT, true>(b, stream); break;
+    default: return cudaErrorInvalidValue;
+  }
+  if (e != cudaSuccess) return e;
+  b.only_marked = kLpt16Mark2;
+  return launch_replay_lpt(b, policy, stream);
 }
 
 }  // namespace convgpu

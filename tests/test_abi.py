@@ -43,7 +43,7 @@ def test_nm_lists_symbols_as_extern_c(so):
 
 def test_version_and_strerror(so):
     assert so.convgpu_abi_version() == 4
-    assert so.convgpu_launches_per_call() == 2
+    assert so.convgpu_launches_per_call() == 3
     assert b"invalid" in so.convgpu_strerror(-errno.EINVAL)
     assert b"sm_100" in so.convgpu_strerror(-errno.ENODEV)
 
@@ -63,7 +63,7 @@ def _traces(**kw):
 
 @pytest.mark.parametrize("kw", [dict(n_containers=0), dict(n_containers=65), dict(n_ops=0),
                                 dict(n_ops=9), dict(arrival=None), dict(op_arg=None),
-                                dict(kernel_variant=4), dict(ctx_overhead_mib=1 << 30),
+                                dict(kernel_variant=5), dict(ctx_overhead_mib=1 << 30),
                                 dict(kernel_variant=3, n_containers=16)])
 def test_replay_rejects_bad_shape_before_touching_the_device(so, kw):
     out = cg.OutT()
@@ -133,7 +133,7 @@ def _traces16(**kw):
 
 
 @pytest.mark.parametrize("kw", [dict(n_ops=5), dict(n_ops=0), dict(n_containers=65),
-                                dict(op_kinds=None), dict(arrival=None), dict(kernel_variant=4)])
+                                dict(op_kinds=None), dict(arrival=None), dict(kernel_variant=5)])
 def test_replay_host16_rejects_bad_shape_before_touching_the_device(so, kw):
     st = (C.c_uint8 * 96)()
     assert so.convgpu_replay_host16(C.byref(_traces16(**kw)), 10, 1000, 1, None, st, 1, 1 << 30,

@@ -1,7 +1,7 @@
 """GPU parity of the compact lane-per-trace kernel (csrc/replay_lpt16.cu,
 CONVGPU_KERNEL_LANE_COMPACT) against the C oracle, element by element, on
 every integer output: configs [2] and [4] (rho 8 has limits above the 16-bit
-fields, so its traces go through the marked 32-bit fallback launch), edge-case
+fields, so its traces go through the marked 17-bit second launch), edge-case
 batches with tiny deltas (consecutive events of one container hit the
 register-fetch slow path), extreme values (fallback and static flags), a
 batch mixing eligible and ineligible traces, and the full-size config [2]
@@ -42,9 +42,10 @@ def test_lane16_rho_sweep(cg, orc, policy, rho):
     w = W.rho_sweep(rho, rand_seed=rho * 7 + 1)
     ref = orc.replay_range(w, policy, 10_000, 11_500, full=True)
     tr = cg.generate(w.gen, 10_000, 1_500)
-    out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel="lane16")
-    _compare(cg, out, ref)
-    _compare_stats(cg, out, ref["stats"])
+    for kernel in ("lane16", "lane16w"):
+        out = _gpu_replay(cg, tr, w.cap, policy, seed=w.rand_seed, kernel=kernel)
+        _compare(cg, out, ref)
+        _compare_stats(cg, out, ref["stats"])
 
 
 EDGE64 = [  # (cap, ovh, mode, count)
@@ -227,19 +228,21 @@ def test_lane16_summary_only_with_scratch(cg, orc, policy):
 @pytest.mark.parametrize("policy", POLS)
 def test_lane16_scratch_reuse_clears_stale_marks(cg, orc, policy):
     """A scratch buffer reused across calls: the first call leaves fallback
-    marks (rho = 8 limits exceed the 16-bit fields) in the slots that the
-    second call's statically flagged traces never write; those traces must
-    not be replayed a second time by the fallback pass."""
+    marks (deltas above 16 bits: neither compact layout holds them) in the
+    scratch; the second call's traces must not be replayed a second time by a
+    fallback pass."""
     import torch
-    w8 = W.rho_sweep(8, rand_seed=1)
     N = 512
-    tr8 = cg.generate(w8.gen, 0, N)
+    b0 = W.random_batch(5, N, 64, 4, 200, mode="valid", limit_choices=range(0, 201))
+    delta = b0.delta.copy()
+    delta[::2, 1, 0] = 0x10000
+    tr0 = cg.traces_from_numpy(b0.arrival, b0.limit, delta, b0.arg)
     scratch = torch.empty(N, 64, dtype=torch.int32, device="cuda")
     out = cg.alloc_out(N, 64, full=False, scratch=False)
     out.admit_scratch = scratch
-    cg.replay(tr8, w8.cap, policy, out, rand_seed=1, kernel="lane16")
+    cg.replay(tr0, 200, policy, out, rand_seed=1, kernel="lane16")
     torch.cuda.synchronize()
-    assert (scratch[:, 0].cpu().numpy().view(np.uint32) == 0xFFFFFFFE).any()
+    assert (scratch[:, 0].cpu().numpy().view(np.uint32) == 0xFFFFFFFD).any()
     b = W.random_batch(3, N, 64, 4, 200, mode="biglimit", limit_choices=range(0, 201))
     tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg)
     ref = orc.replay_batch(b, 200, policy)
@@ -406,3 +409,71 @@ def test_lane16_field_boundaries(cg, orc, policy):
         _compare_stats(cg, out, ref["stats"])
     flags = ref["flags"]
     assert (flags & (1 << 5)).any() and (flags == 0).sum() > 20  # TICK_RANGE present, most valid
+
+
+def _wide_batch(seed):
+    """Traces for the compact kernel's 17-bit pass (limits above 0xFFFE): per
+    trace i, by i % 8, a few containers get
+      0: nothing (16-bit layout)
+      1: limit 0x1FFFF, ALLOC 0xFFFE, ALLOC 0xFFFE, FREE 0xFFFE (used reaches
+         0x1FFFE with the context charge: the 17-bit used field)
+      2: limit 0x10000, ALLOC 0x8000, ALLOC 0x7FFE, FREE 0x8000 (17-bit)
+      3: as 1 with a second ALLOC of 0xFFFF (a size above 16 bits: 32-bit pass)
+      4: limit 0x20000 (above 17 bits: 32-bit pass)
+      5: as 1 with FREE 0xFFFF (32-bit pass)
+      6: limit 0x18000, ALLOC 0xFFFE, ALLOC 0xFFFE (the second rejected), FREE
+         0x100 (17-bit)
+      7: limit 0x1FFFF, first op a FREE of 0xFFFE (INVALID_FREE, 17-bit)
+    on a capacity of 0x30000 MiB (the large containers contend), ovh 2."""
+    n, K, cap, ovh = 64, 4, 0x30000, 2
+    rng = np.random.default_rng(seed)
+    # at most 5 distinct limits per trace: Best-Fit's class rule keeps the
+    # trace in the compact kernel
+    b = W.random_batch(seed, 64, n, K, cap, ovh=ovh, mode="valid", limit_choices=[300, 4000, 9000, 17000])
+    limit, arg = b.limit.copy(), b.arg.copy()
+    A, F, X = W.ALLOC, W.FREE, W.FINISH
+    progs = {1: (0x1FFFF, [(A, 0xFFFE), (A, 0xFFFE), (F, 0xFFFE)]),
+             2: (0x10000, [(A, 0x8000), (A, 0x7FFE), (F, 0x8000)]),
+             3: (0x1FFFF, [(A, 0xFFFE), (A, 0xFFFF), (F, 0xFFFE)]),
+             4: (0x20000, [(A, 0xFFFE), (A, 0xFFFE), (F, 0xFFFE)]),
+             5: (0x1FFFF, [(A, 0xFFFE), (A, 0xFFFE), (F, 0xFFFF)]),
+             6: (0x18000, [(A, 0xFFFE), (A, 0xFFFE), (F, 0x100)]),
+             7: (0x1FFFF, [(F, 0xFFFE), (A, 0x10), (A, 0x10)])}
+    for i in range(64):
+        kind = i % 8
+        if kind == 0:
+            continue
+        L, prog = progs[kind]
+        for c in rng.choice(n, size=6, replace=False):
+            limit[i, c] = L
+            for k, (kk, sz) in enumerate(prog):
+                arg[i, k, c] = W.op(kk, sz)
+            arg[i, 3, c] = W.op(X)
+    return W.Batch(n, K, b.arrival, limit, b.delta, arg), cap, ovh
+
+
+@pytest.mark.parametrize("policy", POLS)
+def test_lane16_wide_pass(cg, orc, policy):
+    """The 17-bit second pass of the compact kernel against the oracle,
+    element by element (every kernel variant), and its routing: after a
+    summary-only compact replay, exactly the traces the 17-bit layout cannot
+    hold carry the second mark (0xFFFFFFFD) in their scratch slot."""
+    import torch
+    b, cap, ovh = _wide_batch(4242)
+    ref = orc.replay_batch(b, cap, policy, tid_base=9, rand_seed=3, ovh=ovh)
+    tr = cg.traces_from_numpy(b.arrival, b.limit, b.delta, b.arg, trace_id_base=9)
+    for kernel, full in (("lane16", True), ("lane16", False), ("lane16w", True), ("lane16w", False),
+                         ("auto", True), ("lane", True), ("warp", True)):
+        out = _gpu_replay(cg, tr, cap, policy, seed=3, ovh=ovh, kernel=kernel, full=full)
+        _compare(cg, out, ref, full=full)
+        _compare_stats(cg, out, ref["stats"])
+    scratch = torch.zeros(64, 64, dtype=torch.int32, device="cuda")
+    out = cg.alloc_out(64, 64, full=False, scratch=False)
+    out.admit_scratch = scratch
+    cg.replay(tr, cap, policy, out, rand_seed=3, ovh=ovh, kernel="lane16")
+    torch.cuda.synchronize()
+    m2 = scratch[:, 0].cpu().numpy().view(np.uint32) == 0xFFFFFFFD
+    kinds = np.arange(64) % 8
+    np.testing.assert_array_equal(m2, np.isin(kinds, [3, 4, 5]))
+    assert (ref["flags"][kinds == 7] & (1 << 3)).all()  # INVALID_FREE on the 17-bit pass
+    assert ref["stats"]["n_rejected"] > 0
