@@ -386,6 +386,7 @@ int host_replay(const convgpu_traces_t* t32, const convgpu_traces16_t* t16, uint
       convgpu::ReplayArgs a = make_args(&dt, cnt, cap);
       a.summary = host_summary ? sum[b][q] : nullptr;
       a.adm_scratch = adm_scratch + (size_t)q * l.cn / 4;  // admissions only
+      a.no_wide = packed;  // 16-bit limits: no 17-bit pass (replay_lpt16.cu)
       a.stats = (convgpu_stats_t*)((char*)dstats + q * stb);
       if (e == cudaSuccess) e = launch_any(a, pols[q], ht.kernel_variant, ps[q]);
       if (e == cudaSuccess) e = cudaEventRecord(pdone[q], ps[q]);

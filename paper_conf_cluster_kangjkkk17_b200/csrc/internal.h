@@ -29,6 +29,7 @@ struct ReplayArgs {
   uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
   uint32_t only_marked;    // 0, or a mark: replay only traces with adm_buf()[i*n] == only_marked
   uint32_t* adm_scratch;   // compact kernel: admissions during the replay when admit_tick == NULL
+  uint32_t no_wide;        // compact kernel: no 17-bit pass (16-bit host format: limits <= 0xFFFF)
 
   // where the compact kernel keeps admissions (and its fallback marks)
   __host__ __device__ uint32_t* adm_buf() const { return admit_tick ? admit_tick : adm_scratch; }

@@ -55,18 +55,18 @@ using lpt::shl_c;
 using lpt::sts_if;
 
 constexpr uint32_t N = 64, KOPS = 4;  // compile-time shape (configs [2]-[4])
-// ust word: used (16 bits; WIDE: 17) | op index 3 | FIRST | PAUSED | ADMITTED |
-// op kinds 2 x K (| WIDE: bit 16 of the declared limit, whose bits 0-15 are
-// in the u16 limit array)
+// ust word: used (16 bits; WIDE: 17) | op index 2 (K = 4: 0..3, FINISH is op
+// 3) | FIRST | PAUSED | ADMITTED | op kinds 2 x K | WIDE: bit 16 of the
+// declared limit, whose bits 0-15 are in the u16 limit array
 template <bool WIDE>
 struct Lay {
   static constexpr uint32_t kUsedBits = WIDE ? 17u : 16u;
   static constexpr uint32_t kUsedMask = (1u << kUsedBits) - 1u;
   static constexpr uint32_t kKShift = kUsedBits;
-  static constexpr uint32_t kFirst = 1u << (kUsedBits + 3);
-  static constexpr uint32_t kPaused = 1u << (kUsedBits + 4);
-  static constexpr uint32_t kAdmitted = 1u << (kUsedBits + 5);
-  static constexpr uint32_t kKindShift = kUsedBits + 6;
+  static constexpr uint32_t kFirst = 1u << (kUsedBits + 2);
+  static constexpr uint32_t kPaused = 1u << (kUsedBits + 3);
+  static constexpr uint32_t kAdmitted = 1u << (kUsedBits + 4);
+  static constexpr uint32_t kKindShift = kUsedBits + 5;
   static constexpr uint32_t kLimHi = WIDE ? 1u << 31 : 0u;
 };
 // keys
@@ -523,7 +523,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             events += fz ? 1u : 0u;
             const uint32_t ust1 = arr ? ((vadm ? kAdmitted : 0u) | (ust & (kKindsMask | kLimHi))) : ust;
             const uint32_t tg1 = vtgt ? c : target;
-            const uint32_t k = (ust1 >> kKShift) & 7u;
+            const uint32_t k = (ust1 >> kKShift) & 3u;
             const uint32_t kind = (ust1 >> (kKindShift + 2 * k)) & 3u;
             const uint32_t r = sd & 0xFFFFu, used = ust1 & kUsedMask;
             const uint32_t nd = (arr && !fz) ? (ust & kUsedMask) : (sd >> 16);  // d_0 / d_{k+1}
@@ -672,7 +672,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
             uint32_t nu = res ? (((ut & ~(kUsedMask | kPaused)) | (uu + pend) | kFirst) + kKOne) : ut;
             nu |= full ? kAdmitted : 0u;
             nkc = ((t + (sdt >> 16)) << 6) | tg;
-            pfk = res ? ((nu >> kKShift) & 7u) : 0xFFu;
+            pfk = res ? ((nu >> kKShift) & 3u) : 0xFFu;
             AT(s_ust, tg) = nu;
             const uint32_t rmask = res ? 0xFFFFFFFFu : 0u;
             pm_lo &= ~(shl_c(1u, tg) & rmask);
@@ -832,6 +832,9 @@ cudaError_t launch_replay_lpt16(const ReplayArgs& a, int policy, cudaStream_t st
   // R1-LIT: the traces the 16-bit layout cannot hold go to the warp-per-trace
   // kernel (which implements that reading), marked only
   if (lit) return launch_replay(b, policy, false, stream);
+  // 16-bit host format (limits <= 0xFFFF): the 17-bit pass could only take
+  // limits of exactly 0xFFFF; the 32-bit kernel does, one launch fewer
+  if (a.no_wide) return launch_replay_lpt(b, policy, stream);
   // R1: to the 17-bit layout (WIDE), marked only; what that cannot hold
   // either (re-marked kLpt16Mark2) to the 32-bit lane kernel
 #ifdef LPT16_NO_WIDE

@@ -13,6 +13,7 @@ total and mean device time, share of the listed time).
 """
 import argparse
 import csv
+import re
 import io
 import json
 import os
@@ -45,11 +46,13 @@ def raw(rep):
     return rows[0], rows[1], rows[2:]
 
 
-def full(rep, tag, events_per_launch, traffic, workload, traces):
+def full(rep, tag, events_per_launch, traffic, workload, traces, only=None):
     hdr, units, data = raw(rep)
     idx = {h: i for i, h in enumerate(hdr)}
     kernels = []
     for r in data:
+        if only and not re.search(only, r[idx["Kernel Name"]]):
+            continue
         k = {"kernel": r[idx["Kernel Name"]]}
         for key in KEYS:
             if key in idx:
@@ -116,10 +119,12 @@ def main():
     ap.add_argument("--traffic", action="store_true")
     ap.add_argument("--workload", default="c2_1e6x64_rho2")
     ap.add_argument("--traces", type=int, default=1_000_000)
+    ap.add_argument("--only", default=None, help="regex: summarise only these kernels (e.g. the "
+                    "compact kernel's first pass, not its 17-bit / 32-bit fallback passes)")
     a = ap.parse_args()
     os.makedirs(PROF, exist_ok=True)
     if a.rep:
-        full(a.rep, a.tag, a.events, a.traffic, a.workload, a.traces)
+        full(a.rep, a.tag, a.events, a.traffic, a.workload, a.traces, a.only)
     if a.launches:
         launches(a.launches, a.tag)
 
