@@ -475,6 +475,76 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     }
   };
 
+  // SELECT (R3-R7): a new fill target when there is none (FIFO:
+  // computed unconditionally, taken by lanes with `on`)
+  auto select_target = [&](bool on) {
+    if (P == CONVGPU_FIFO) {
+      const bool ns = on && target == kNoC;  // (always under R1-LIT: no sticky target)
+      const uint32_t sel = ffs64(pm_lo, pm_hi);
+      target = ns ? sel : target;
+      a_tg = ns ? (LIT ? (uint32_t)ASG(sel & 63u) : 0u) : a_tg;  // R1-LIT: its partial hold
+      n_sel += ns ? 1u : 0u;
+    } else if (on && target == kNoC) {
+      uint32_t sel;
+      if (P == CONVGPU_BEST_FIT && LIT) {  // R3, R4 with partial holds: shortfall L - a
+        uint32_t best = kNoC, bneed = 0, mn = kNoC, mneed = 0xFFFFFFFFu;
+        uint32_t wl = pm_lo, wh = pm_hi;
+        while (wl | wh) {  // ascending index: strict comparisons keep the lowest
+          const uint32_t c = ffs64(wl, wh);
+          wl &= ~shl_c(1u, c);
+          wh &= ~shl_c(1u, c - 32u);
+          const uint32_t need = (uint32_t)LIM(c) - (uint32_t)ASG(c);
+          const bool f = need <= free_mem && (best == kNoC || need > bneed);
+          best = f ? c : best;
+          bneed = f ? need : bneed;
+          const bool m = need < mneed;
+          mn = m ? c : mn;
+          mneed = m ? need : mneed;
+        }
+        sel = best != kNoC ? best : mn;
+      } else if (P == CONVGPU_BEST_FIT) {  // R3, R4 (classes: see bl above)
+        // ascending classes: the last fitting class with a paused
+        // member wins; descending: the last class with one is the lowest
+        uint32_t fl = 0, fh = 0, ml = 0, mh = 0;
+#pragma unroll
+        for (int j = 0; j < kBfClasses; ++j) {
+          const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
+          const bool on = ((a | b) != 0u) && bl[j] <= free_mem;
+          fl = on ? a : fl;
+          fh = on ? b : fh;
+        }
+#pragma unroll
+        for (int j = kBfClasses - 1; j >= 0; --j) {
+          const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
+          const bool on = (a | b) != 0u;
+          ml = on ? a : ml;
+          mh = on ? b : mh;
+        }
+        const bool fit = (fl | fh) != 0u;
+        sel = ffs64(fit ? fl : ml, fit ? fh : mh);
+      } else if (P == CONVGPU_RECENT_FIT) {  // R5
+        // pop the suspension stack: paused containers leave the paused
+        // set only by resuming, and only the target resumes, so popping
+        // at selection keeps the stack exactly the paused set in
+        // suspension order.  R1-LIT: the selected container may stay
+        // paused (partially filled), so it is popped when it resumes
+        sel = ru_head;
+        if (!LIT) ru_head = AT(s_key, sel) & 127u;
+      } else {  // RANDOM_FIT (R6)
+        const uint64_t tid = p.tid_base + i;
+        const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
+        const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
+                                   (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
+        ++draws;
+        const uint32_t jj = __umulhi(x.x, m);
+        sel = lpt::nth_set64(pm_lo, pm_hi, jj);
+      }
+      target = sel;
+      a_tg = LIT ? (uint32_t)ASG(sel) : 0u;  // R1-LIT: its partial hold
+      ++n_sel;
+    }
+  };
+
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
   if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; }
@@ -587,71 +657,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         } else if (dmode) {
           // ====== one DISPATCH step at the triggering tick (R1, R9) ======
           const uint32_t t = cur_t;
-          if (P == CONVGPU_FIFO) {
-            const bool ns = target == kNoC;  // (always under R1-LIT: no sticky target)
-            const uint32_t sel = ffs64(pm_lo, pm_hi);
-            target = ns ? sel : target;
-            a_tg = ns ? (LIT ? (uint32_t)ASG(sel & 63u) : 0u) : a_tg;  // R1-LIT: its partial hold
-            n_sel += ns ? 1u : 0u;
-          } else if (target == kNoC) {
-            uint32_t sel;
-            if (P == CONVGPU_BEST_FIT && LIT) {  // R3, R4 with partial holds: shortfall L - a
-              uint32_t best = kNoC, bneed = 0, mn = kNoC, mneed = 0xFFFFFFFFu;
-              uint32_t wl = pm_lo, wh = pm_hi;
-              while (wl | wh) {  // ascending index: strict comparisons keep the lowest
-                const uint32_t c = ffs64(wl, wh);
-                wl &= ~shl_c(1u, c);
-                wh &= ~shl_c(1u, c - 32u);
-                const uint32_t need = (uint32_t)LIM(c) - (uint32_t)ASG(c);
-                const bool f = need <= free_mem && (best == kNoC || need > bneed);
-                best = f ? c : best;
-                bneed = f ? need : bneed;
-                const bool m = need < mneed;
-                mn = m ? c : mn;
-                mneed = m ? need : mneed;
-              }
-              sel = best != kNoC ? best : mn;
-            } else if (P == CONVGPU_BEST_FIT) {  // R3, R4 (classes: see bl above)
-              // ascending classes: the last fitting class with a paused
-              // member wins; descending: the last class with one is the lowest
-              uint32_t fl = 0, fh = 0, ml = 0, mh = 0;
-#pragma unroll
-              for (int j = 0; j < kBfClasses; ++j) {
-                const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
-                const bool on = ((a | b) != 0u) && bl[j] <= free_mem;
-                fl = on ? a : fl;
-                fh = on ? b : fh;
-              }
-#pragma unroll
-              for (int j = kBfClasses - 1; j >= 0; --j) {
-                const uint32_t a = pm_lo & bm_lo[j], b = pm_hi & bm_hi[j];
-                const bool on = (a | b) != 0u;
-                ml = on ? a : ml;
-                mh = on ? b : mh;
-              }
-              const bool fit = (fl | fh) != 0u;
-              sel = ffs64(fit ? fl : ml, fit ? fh : mh);
-            } else if (P == CONVGPU_RECENT_FIT) {  // R5
-              // pop the suspension stack: paused containers leave the paused
-              // set only by resuming, and only the target resumes, so popping
-              // at selection keeps the stack exactly the paused set in
-              // suspension order.  R1-LIT: the selected container may stay
-              // paused (partially filled), so it is popped when it resumes
-              sel = ru_head;
-              if (!LIT) ru_head = AT(s_key, sel) & 127u;
-            } else {  // RANDOM_FIT (R6)
-              const uint64_t tid = p.tid_base + i;
-              const uint32_t clo = __popc(pm_lo), m = clo + __popc(pm_hi);
-              const U4 x = philox4x32_10((uint32_t)tid, (uint32_t)(tid >> 32), draws, 1u,
-                                         (uint32_t)p.seed, (uint32_t)(p.seed >> 32));
-              ++draws;
-              const uint32_t jj = __umulhi(x.x, m);
-              sel = lpt::nth_set64(pm_lo, pm_hi, jj);
-            }
-            target = sel;
-            a_tg = LIT ? (uint32_t)ASG(sel) : 0u;  // R1-LIT: its partial hold
-            ++n_sel;
-          }
+          select_target(true);
           {
             // the target was not fetched in the previous iteration: a dispatch
             // step follows a pause / FINISH (no fetch) or an admission, after
