@@ -103,7 +103,13 @@ __device__ __forceinline__ void tmem_fence_before_sync() {
 __device__ __forceinline__ void tmem_fence_after_sync() {
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
 }
-// 16 consecutive columns of this thread's lane
+// 16 consecutive columns of this thread's lane.  No "memory" clobber: TMEM is
+// not generic memory, so global / shared accesses may be scheduled across the
+// store (init's loads of the next containers overlap it); tcgen05.wait::st and
+// the volatile loads keep TMEM ordered.
+#ifndef TMEM_ST_CLOBBER
+#define TMEM_ST_CLOBBER
+#endif
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* v) {
   asm volatile(
       "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
@@ -111,7 +117,7 @@ __device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* v) {
       ::"r"(taddr), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]),
         "r"(v[7]), "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]),
         "r"(v[14]), "r"(v[15])
-      : "memory");
+      TMEM_ST_CLOBBER);
 }
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
   asm volatile(
@@ -122,6 +128,19 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* v) {
         "=r"(v[14]), "=r"(v[15])
       : "r"(taddr)
       : "memory");
+}
+// 16-byte global loads issued exactly where written (volatile: the compiler
+// may not sink them to their first use, so a batch of them is in flight
+// together), cached at L2 only (.cg): one warp's 32 traces are 32 different
+// lines per load, so L1 (what shared memory leaves of it) cannot hold them,
+// while L2 keeps the rows for the event loop's op fetches.  Measured on the
+// compact kernel's init: .cg 4.31, .nc 4.24, .ca 4.22, .cs (evict-first) 3.28
+// x 10^10 events/s.
+__device__ __forceinline__ uint4 ldg4_cg(const void* p) {
+  uint4 v;
+  asm volatile("ld.global.cg.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  return v;
 }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }

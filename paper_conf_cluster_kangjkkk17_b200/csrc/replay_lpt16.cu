@@ -272,12 +272,27 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     uint32_t bad = 0, lsum = 0, amax = 0, prev = 0, lmax = 0, dmax = 0, smax = 0;
 #pragma unroll
     for (int j = 0; j < 8; ++j) gmin[j] = kKeyNone;
+    // two-stage software pipeline: the loads of containers 4q+4..4q+7 are in
+    // flight while 4q..4q+3 are processed (one warp's 32 traces are 32
+    // separate rows per load)
+    uint4 a4b[2], l4b[2], d4b[2][4], w4b[2][4];
+    auto ld_q = [&](uint32_t q, int s) {
+      a4b[s] = lpt::ldg4_cg(A4 + q);
+      l4b[s] = lpt::ldg4_cg(L4 + q);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        d4b[s][k] = lpt::ldg4_cg(D4 + k * 16 + q);
+        w4b[s][k] = lpt::ldg4_cg(R4 + k * 16 + q);
+      }
+    };
+    ld_q(0, 0);
 #pragma unroll
     for (uint32_t q = 0; q < 16; ++q) {
-      const uint4 a4 = __ldg(A4 + q), l4 = __ldg(L4 + q);
+      if (q + 1 < 16) ld_q(q + 1, (q + 1) & 1);
+      const uint4 a4 = a4b[q & 1], l4 = l4b[q & 1];
       uint4 d4[4], w4[4];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) { d4[k] = __ldg(D4 + k * 16 + q); w4[k] = __ldg(R4 + k * 16 + q); }
+      for (int k = 0; k < 4; ++k) { d4[k] = d4b[q & 1][k]; w4[k] = w4b[q & 1][k]; }
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const uint32_t c = 4 * q + j, a = comp(a4, j), L = comp(l4, j);
@@ -393,6 +408,11 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     uint32_t mfin = 0;
     const uint64_t ob = ti * n;
     const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
+    // all 16 admission loads in flight at once (this thread stored them during
+    // the replay: read at L2), then the parked sums
+    uint4 m4a[16];
+#pragma unroll
+    for (uint32_t q = 0; q < 16; ++q) m4a[q] = lpt::ldg4_cg(M4 + q);
 #pragma unroll
     for (uint32_t q = 0; q < 16; ++q) {
       if ((q & 3) == 0) {  // the next 16 parked sums
@@ -401,7 +421,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         lpt::tmem_wait_ld();
       }
       // admissions this thread stored during the replay (coherent load)
-      const uint4 m4 = stopped ? make_uint4(0, 0, 0, 0) : M4[q];
+      const uint4 m4 = stopped ? make_uint4(0, 0, 0, 0) : m4a[q];
       uint32_t at[4], ar[4], wt[4], fn[4];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -547,7 +567,12 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
 
   bool have = i < p.count, tdone = false, dmode = false;
   uint32_t cur_t = 0;
-  if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; }
+#ifdef LPT16_NOLOOP  // experiment: init + epilogue only
+#define LPT16_TD true
+#else
+#define LPT16_TD (flags != 0 || skip)
+#endif
+  if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = LPT16_TD; }
   park_state();
   while (__any_sync(kFull, have)) {
     do {
@@ -724,7 +749,10 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       i = next(i + T);
       have = i < p.count;
     }
-    if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = flags != 0 || skip; dmode = false; }
+#ifdef LPT16_INIT2  // experiment: init twice (its cost in the running kernel)
+    if (__any_sync(kFull, have)) { init(have ? i : 0, have); }
+#endif
+    if (__any_sync(kFull, have)) { init(have ? i : 0, have); tdone = LPT16_TD; dmode = false; }
     park_state();
   }
   fetch_state();  // the statistics accumulators, for the final reduction
