@@ -13,6 +13,7 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/$
 timeout 600 python bench.py --workload c1 --no-cpu-baseline > gpurun_out/${T}_bench_c1.json 2> gpurun_out/${T}_bench_c1.err; echo c1=$?
 timeout 600 python bench.py --workload mimic --no-cpu-baseline > gpurun_out/${T}_bench_mimic.json 2> gpurun_out/${T}_bench_mimic.err; echo mimic=$?
 timeout 900 python bench.py --workload c3 --steps 2 --warmup 1 > gpurun_out/${T}_bench_c3.json 2> gpurun_out/${T}_bench_c3.err; echo c3=$?
+timeout 900 python scripts/rho_sweep.py --out gpurun_out/${T}_rho_sweep.json > gpurun_out/${T}_rho_sweep.txt 2>&1; echo rho=$?
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches.csv python bench.py --steps 3 --warmup 3 --profile > gpurun_out/ncu_launch_bench.log 2>&1; echo ncu_launch=$?
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:replay_lpt16 -c 8 -o gpurun_out/${T}_prof python bench.py --steps 1 --warmup 1 --profile > gpurun_out/ncu_full.log 2>&1; echo ncu_full=$?
 ls -la gpurun_out
