@@ -52,6 +52,17 @@ tr8 = cg.traces_from_numpy(b8.arrival, b8.limit, b8.delta, b8.arg)
 cg.replay(tr8, 256, "best_fit", cg.alloc_out(300, 64), kernel="lane16")
 w4 = W.rho_sweep(8, rand_seed=3)
 tr4 = cg.generate(w4.gen, 0, 300)
+# the 17-bit layout as the first pass (rho 8) and a batch whose deltas exceed
+# 16 bits (marked by the 16-bit and the 17-bit passes, replayed by the 32-bit)
+for pol in W.POLICIES:
+    cg.replay(tr4, w4.cap, pol, cg.alloc_out(300, 64), rand_seed=3, kernel="lane16w")
+    cg.replay(tr4, w4.cap, pol, cg.alloc_out(300, 64, full=False), rand_seed=3, kernel="lane16w")
+bd = W.random_batch(8, 300, 64, 4, 200, mode="valid", limit_choices=range(0, 201))
+dd = bd.delta.copy()
+dd[::3, 1, 0] = 0x10000
+trd = cg.traces_from_numpy(bd.arrival, bd.limit, dd, bd.arg)
+for pol in W.POLICIES:
+    cg.replay(trd, 200, pol, cg.alloc_out(300, 64), kernel="lane16")
 for pol in W.POLICIES:
     cg.replay(tr4, w4.cap, pol + "+literal", cg.alloc_out(300, 64), rand_seed=3, kernel="lane16")
 torch.cuda.synchronize()
