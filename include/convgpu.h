@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define CONVGPU_ABI_VERSION 4
+#define CONVGPU_ABI_VERSION 5  /* 5: CONVGPU_KERNEL_LANE_COMPACT_WIDE */
 #define CONVGPU_MAX_CONTAINERS 64u   /* containers per trace */
 #define CONVGPU_MAX_OPS 8u           /* ops per container (K) */
 #define CONVGPU_CAPACITY_LIMIT (1u << 26) /* capacity_mib must be below this */

@@ -42,7 +42,7 @@ def test_nm_lists_symbols_as_extern_c(so):
 
 
 def test_version_and_strerror(so):
-    assert so.convgpu_abi_version() == 4
+    assert so.convgpu_abi_version() == 5
     assert so.convgpu_launches_per_call() == 3
     assert b"invalid" in so.convgpu_strerror(-errno.EINVAL)
     assert b"sm_100" in so.convgpu_strerror(-errno.ENODEV)

@@ -477,3 +477,25 @@ def test_lane16_wide_pass(cg, orc, policy):
     np.testing.assert_array_equal(m2, np.isin(kinds, [3, 4, 5]))
     assert (ref["flags"][kinds == 7] & (1 << 3)).all()  # INVALID_FREE on the 17-bit pass
     assert ref["stats"]["n_rejected"] > 0
+
+
+@pytest.mark.parametrize("kernel", ["lane16", "lane16w"])
+def test_lane16_host_path_wide(cg, orc, kernel):
+    """The 32-bit host path (convgpu_replay_host) on config [4] at rho = 8
+    (limits above 16 bits) with the compact kernel's 16-bit-first and
+    17-bit-first chains: every trace's summary and the statistics of all four
+    policies against the oracle."""
+    w = W.rho_sweep(8, rand_seed=11)
+    base, N = 70_000, 2 * 4096 + 777
+    A, L, D, R = orc.generate_batch(w.gen, base, N)
+    summ = np.zeros((4, N), cg.SUMMARY_DTYPE)
+    st = cg.replay_host(A, L, D, R, w.cap, POLS, trace_id_base=base, summary=summ,
+                        rand_seed=11, chunk=4096, kernel=kernel)
+    for q, pol in enumerate(POLS):
+        ref = orc.replay_range(w, pol, base, base + N)
+        for f in ("makespan", "peak_reserved", "peak_used", "flags", "sum_wait", "n_rejected",
+                  "n_select", "digest"):
+            np.testing.assert_array_equal(summ[q][f], ref[f].astype(summ[q][f].dtype),
+                                          err_msg=f"{pol} {f}")
+        for k, v in ref["stats"].items():
+            assert cg.stats_dict(st[q])[k] == v, (pol, k)
