@@ -78,6 +78,8 @@ convgpu::ReplayArgs make_args(const convgpu_traces_t* t, uint64_t n, uint32_t ca
   return a;
 }
 
+bool aligned32(const void* p) { return ((uintptr_t)p & 31u) == 0; }
+
 bool use_bulk(const convgpu::ReplayArgs& a) {
   return (a.n % 4u) == 0 && aligned16(a.arrival) && aligned16(a.limit) && aligned16(a.delta) &&
          aligned16(a.arg);
@@ -101,6 +103,10 @@ uint32_t auto_variant(uint64_t count, int policy) {
 cudaError_t launch_any(convgpu::ReplayArgs a, int policy, uint32_t variant, cudaStream_t s) {
   a.aligned16 = use_bulk(a) && aligned16(a.admit_tick) && aligned16(a.adm_scratch) &&
                 aligned16(a.wait) && aligned16(a.finish) && ((uintptr_t)a.admit_rank & 3u) == 0;
+  // 32-byte loads of the trace and the admissions, 32-byte output stores
+  a.aligned32 = (a.n % 8u) == 0 && aligned32(a.arrival) && aligned32(a.limit) && aligned32(a.delta) &&
+                aligned32(a.arg) && aligned32(a.admit_tick) && aligned32(a.adm_scratch) &&
+                aligned32(a.wait) && aligned32(a.finish) && ((uintptr_t)a.admit_rank & 7u) == 0;
   if (variant == CONVGPU_KERNEL_AUTO) {
     variant = auto_variant(a.count, policy);
     if (variant == CONVGPU_KERNEL_LANE_PER_TRACE && convgpu::lpt16_supported(a))

@@ -27,6 +27,7 @@ struct ReplayArgs {
   uint64_t grid_override;  // 0 = occupancy-sized persistent grid
   uint32_t per_sm_cap;     // tuning knob (env CONVGPU_PER_SM_CAP): at most this many CTAs per SM
   uint32_t aligned16;      // all trace arrays and per-container outputs 16-B aligned, n % 4 == 0
+  uint32_t aligned32;      // the four trace arrays 32-B aligned and n % 8 == 0 (32-byte loads)
   uint32_t only_marked;    // 0, or a mark: replay only traces with adm_buf()[i*n] == only_marked
   uint32_t* adm_scratch;   // compact kernel: admissions during the replay when admit_tick == NULL
   uint32_t no_wide;        // compact kernel: no 17-bit pass (16-bit host format: limits <= 0xFFFF)

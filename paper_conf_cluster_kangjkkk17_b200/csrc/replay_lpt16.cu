@@ -58,6 +58,9 @@ constexpr uint32_t N = 64, KOPS = 4;  // compile-time shape (configs [2]-[4])
 // ust word: used (16 bits; WIDE: 17) | op index 2 (K = 4: 0..3, FINISH is op
 // 3) | FIRST | PAUSED | ADMITTED | op kinds 2 x K | WIDE: bit 16 of the
 // declared limit, whose bits 0-15 are in the u16 limit array
+#ifndef LPT16_V8
+#define LPT16_V8 1
+#endif
 template <bool WIDE>
 struct Lay {
   static constexpr uint32_t kUsedBits = WIDE ? 17u : 16u;
@@ -285,50 +288,78 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         w4b[s][k] = lpt::ldg4_cg(R4 + k * 16 + q);
       }
     };
+    // one container's values: validation, derived state, shared-memory words
+    auto proc = [&](uint32_t c, uint32_t a, uint32_t L, const uint32_t (&d)[4], const uint32_t (&w)[4]) {
+      if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
+      if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
+      prev = a;
+      amax = max(amax, a);
+      lmax = max(lmax, L);
+      uint32_t kinds = 0, bsum = a;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        bsum += d[k];
+        lsum = min(lsum + min(d[k], kTickLimit), kTickLimit);
+        dmax = max(dmax, d[k]);
+        if (((w[k] >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
+        if (WIDE && ((w[k] >> 30) == CONVGPU_OP_ALLOC || (w[k] >> 30) == CONVGPU_OP_FREE))
+          smax = max(smax, w[k] & kSizeMask);
+        kinds |= (w[k] >> 30) << (2 * k);
+      }
+      const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
+      AT(s_key, c) = key;
+      AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(d[0], 0xFFFFu) |
+                     (WIDE ? ((L >> 16) & 1u) << 31 : 0u);
+      AT(s_sd, c) = pack_sd(w[0], min(d[1], 0xFFFFu));
+      LIM(c) = (uint16_t)(WIDE ? L : min(L, 0xFFFFu));  // WIDE: bit 16 in the ust word
+      if (LIT) ASG(c) = 0;
+      gmin[c >> 3] = min(gmin[c >> 3], key);
+      base[c & 15] = bsum;
+      if (c == 0) arr0 = a;
+    };
+    if (LPT16_V8 && p.aligned32) {
+    // 32-byte loads (LDG.256: one full sector per lane), 8 containers a step
+    // (the four trace arrays 32-B aligned; warp-uniform)
+#pragma unroll
+    for (uint32_t q = 0; q < 8; ++q) {
+      uint32_t av[8], lv[8], dv[4][8], wv[4][8];
+      lpt::ldg8_cg(av, p.arrival + ti * n + 8 * q);
+      lpt::ldg8_cg(lv, p.limit + ti * n + 8 * q);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        lpt::ldg8_cg(dv[k], trace_delta + k * n + 8 * q);
+        lpt::ldg8_cg(wv[k], trace_arg + k * n + 8 * q);
+      }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const uint32_t d[4] = {dv[0][j], dv[1][j], dv[2][j], dv[3][j]};
+        const uint32_t w[4] = {wv[0][j], wv[1][j], wv[2][j], wv[3][j]};
+        proc(8 * q + j, av[j], lv[j], d, w);
+      }
+      if ((q & 1) == 1) {  // park 16 sums (R17's wait) in this thread's TMEM lane
+        __syncwarp();
+        lpt::tmem_st16(t_base + 8u * (q & ~1u), base);
+      }
+    }
+    } else {
     ld_q(0, 0);
 #pragma unroll
     for (uint32_t q = 0; q < 16; ++q) {
       if (q + 1 < 16) ld_q(q + 1, (q + 1) & 1);
       const uint4 a4 = a4b[q & 1], l4 = l4b[q & 1];
-      uint4 d4[4], w4[4];
-#pragma unroll
-      for (int k = 0; k < 4; ++k) { d4[k] = d4b[q & 1][k]; w4[k] = w4b[q & 1][k]; }
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        const uint32_t c = 4 * q + j, a = comp(a4, j), L = comp(l4, j);
-        if (L > cap) bad |= CONVGPU_FLAG_INVALID_LIMIT;
-        if (c > 0 && a < prev) bad |= CONVGPU_FLAG_UNSORTED_ARRIVAL;
-        prev = a;
-        amax = max(amax, a);
-        lmax = max(lmax, L);
-        uint32_t kinds = 0, bsum = a;
-#pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const uint32_t d = comp(d4[k], j), w = comp(w4[k], j);
-          bsum += d;
-          lsum = min(lsum + min(d, kTickLimit), kTickLimit);
-          dmax = max(dmax, d);
-          if (((w >> 30) == CONVGPU_OP_FINISH) != (k == 3)) bad |= CONVGPU_FLAG_BAD_PROGRAM;
-          if (WIDE && ((w >> 30) == CONVGPU_OP_ALLOC || (w >> 30) == CONVGPU_OP_FREE))
-            smax = max(smax, w & kSizeMask);
-          kinds |= (w >> 30) << (2 * k);
-        }
-        const uint32_t key = (min(a, kTickLimit - 1) << 6) | c;
-        AT(s_key, c) = key;
-        AT(s_ust, c) = kNotArrived | (kinds << kKindShift) | min(comp(d4[0], j), 0xFFFFu) |
-                       (WIDE ? ((L >> 16) & 1u) << 31 : 0u);
-        AT(s_sd, c) = pack_sd(comp(w4[0], j), min(comp(d4[1], j), 0xFFFFu));
-        LIM(c) = (uint16_t)(WIDE ? L : min(L, 0xFFFFu));  // WIDE: bit 16 in the ust word
-        if (LIT) ASG(c) = 0;
-        gmin[c >> 3] = min(gmin[c >> 3], key);
-        base[c & 15] = bsum;
-        if (c == 0) arr0 = a;
+        const uint32_t d[4] = {comp(d4b[q & 1][0], j), comp(d4b[q & 1][1], j), comp(d4b[q & 1][2], j),
+                               comp(d4b[q & 1][3], j)};
+        const uint32_t w[4] = {comp(w4b[q & 1][0], j), comp(w4b[q & 1][1], j), comp(w4b[q & 1][2], j),
+                               comp(w4b[q & 1][3], j)};
+        proc(4 * q + j, comp(a4, j), comp(l4, j), d, w);
       }
       if ((q & 3) == 3) {  // park 16 sums (R17's wait) in this thread's TMEM lane
         __syncwarp();
         lpt::tmem_st16(t_base + 4u * (q & ~3u), base);
       }
-
+    }
     }
     if (amax >= kTickLimit || amax + lsum >= kTickLimit) bad |= CONVGPU_FLAG_TICK_RANGE;
     // not representable in the 16-bit fields: the 32-bit kernel replays it
@@ -407,6 +438,47 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
     uint64_t dig = 0, swait = 0;
     uint32_t mfin = 0;
     const uint64_t ob = ti * n;
+    // one container's outputs and its digest terms
+    auto epi_c = [&](uint32_t c, uint32_t adm, uint32_t bs, uint32_t& at, uint32_t& ar, uint32_t& wt,
+                     uint32_t& fn) {
+      at = kKeyNone; ar = 0xFFu; wt = 0; fn = 0;
+      if (!stopped) {
+        if (AT(s_ust, c) & kAdmitted) {
+          at = adm >> 6;
+          ar = adm & 63u;
+        }
+        fn = AT(s_key, c) & ~kDone;
+        wt = fn - bs;  // R17: wait = finish - arrival - sum of deltas
+      }
+      const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar << 48) ^ (uint64_t)at);
+      dig += mix64(h1 ^ (((uint64_t)wt << 32) | fn));
+      mfin = max(mfin, fn);
+      swait += wt;
+    };
+    if (LPT16_V8 && p.aligned32) {
+      // 32-byte admission loads (all in flight) and 32-byte streaming stores
+      uint32_t m8[8][8];
+#pragma unroll
+      for (uint32_t g = 0; g < 8; ++g) lpt::ldg8_cg(m8[g], adm_out + 8 * g);
+#pragma unroll
+      for (uint32_t g = 0; g < 8; ++g) {
+        if ((g & 1) == 0) {  // the next 16 parked sums
+          __syncwarp();
+          lpt::tmem_ld16(t_base + 8u * g, base);
+          lpt::tmem_wait_ld();
+        }
+        uint32_t at[8], ar[8], wt[8], fn[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+          epi_c(8 * g + j, m8[g][j], base[(8 * g + j) & 15], at[j], ar[j], wt[j], fn[j]);
+        if (act && p.admit_tick) lpt::stg8_cs(p.admit_tick + ob + 8 * g, at);
+        if (act && p.admit_rank)
+          lpt::stg2_cs(p.admit_rank + ob + 8 * g, ar[0] | (ar[1] << 8) | (ar[2] << 16) | (ar[3] << 24),
+                       ar[4] | (ar[5] << 8) | (ar[6] << 16) | (ar[7] << 24));
+        if (act && p.wait) lpt::stg8_cs(p.wait + ob + 8 * g, wt);
+        if (act && p.finish) lpt::stg8_cs(p.finish + ob + 8 * g, fn);
+      }
+    } else {
     const uint4* M4 = reinterpret_cast<const uint4*>(adm_out);
     // all 16 admission loads in flight at once (this thread stored them during
     // the replay: read at L2), then the parked sums
@@ -424,24 +496,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
       const uint4 m4 = stopped ? make_uint4(0, 0, 0, 0) : m4a[q];
       uint32_t at[4], ar[4], wt[4], fn[4];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const uint32_t c = 4 * q + j;
-        at[j] = kKeyNone; ar[j] = 0xFFu; wt[j] = 0; fn[j] = 0;
-        if (!stopped) {
-          if (AT(s_ust, c) & kAdmitted) {
-            const uint32_t adm = comp(m4, j);
-            at[j] = adm >> 6;
-            ar[j] = adm & 63u;
-          }
-          fn[j] = AT(s_key, c) & ~kDone;
-          // R17: wait = finish - arrival - sum of deltas
-          wt[j] = fn[j] - base[c & 15];
-        }
-        const uint64_t h1 = mix64(((uint64_t)c << 56) ^ ((uint64_t)ar[j] << 48) ^ (uint64_t)at[j]);
-        dig += mix64(h1 ^ (((uint64_t)wt[j] << 32) | fn[j]));
-        mfin = max(mfin, fn[j]);
-        swait += wt[j];
-      }
+      for (int j = 0; j < 4; ++j) epi_c(4 * q + j, comp(m4, j), base[(4 * q + j) & 15], at[j], ar[j], wt[j], fn[j]);
       // streaming stores (evict-first): outputs are not re-read, inputs of the
       // traces in flight should stay in L2
       if (act && p.admit_tick)
@@ -453,6 +508,7 @@ __global__ void __launch_bounds__(32 * warps_per_cta(POLICY), 1) replay_lpt16_ke
         __stcs(reinterpret_cast<uint4*>(p.wait + ob) + q, make_uint4(wt[0], wt[1], wt[2], wt[3]));
       if (act && p.finish)
         __stcs(reinterpret_cast<uint4*>(p.finish + ob) + q, make_uint4(fn[0], fn[1], fn[2], fn[3]));
+    }
     }
     const uint32_t makespan = stopped ? 0u : mfin - arr0;
     dig += mix64(((uint64_t)makespan << 32) | peak_res);
