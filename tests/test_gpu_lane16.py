@@ -499,3 +499,50 @@ def test_lane16_host_path_wide(cg, orc, kernel):
                                           err_msg=f"{pol} {f}")
         for k, v in ref["stats"].items():
             assert cg.stats_dict(st[q])[k] == v, (pol, k)
+
+
+def _off16(t, torch):
+    """A contiguous copy of `t` whose data starts 16 bytes past a 32-byte
+    boundary (16-B aligned, not 32-B aligned)."""
+    es = t.element_size()
+    big = torch.empty(t.numel() + 64 // es, dtype=t.dtype, device=t.device)
+    base = big.data_ptr()
+    skip = ((32 - base % 32) % 32 + 16) // es
+    v = big[skip:skip + t.numel()].view(t.shape)
+    v.copy_(t)
+    assert v.data_ptr() % 32 == 16
+    return v
+
+
+@pytest.mark.parametrize("policy", POLS)
+@pytest.mark.parametrize("which", ["traces", "outputs"])
+def test_lane16_16byte_aligned_path(cg, orc, policy, which):
+    """Arrays 16-B but not 32-B aligned take the compact kernel's 16-byte
+    init / epilogue path (the 32-byte one needs every trace array and output
+    32-B aligned): config [2] traces, full outputs and summary-only through
+    the admission scratch, against the oracle."""
+    import torch
+    w = W.CONFIGS["c2"]
+    base, N = 123_456, 5_000
+    tr0 = cg.generate(w.gen, base, N)
+    tr = tr0
+    if which == "traces":
+        tr = cg.Traces(_off16(tr0.arrival, torch), _off16(tr0.limit, torch),
+                       _off16(tr0.op_delta, torch), _off16(tr0.op_arg, torch), base)
+    ref = orc.replay_range(w, policy, base, base + N, full=True)
+    out = cg.alloc_out(N, 64)
+    if which == "outputs":
+        out.admit_tick = _off16(out.admit_tick, torch)
+        out.wait = _off16(out.wait, torch)
+        out.finish = _off16(out.finish, torch)
+    cg.replay(tr, w.cap, policy, out, rand_seed=w.rand_seed, kernel="lane16")
+    torch.cuda.synchronize()
+    _compare(cg, out, ref)
+    _compare_stats(cg, out, ref["stats"])
+    outs = cg.alloc_out(N, 64, full=False)
+    if which == "outputs":
+        outs.admit_scratch = _off16(outs.admit_scratch, torch)
+    cg.replay(tr, w.cap, policy, outs, rand_seed=w.rand_seed, kernel="lane16")
+    torch.cuda.synchronize()
+    _compare(cg, outs, ref, full=False)
+    _compare_stats(cg, outs, ref["stats"])
