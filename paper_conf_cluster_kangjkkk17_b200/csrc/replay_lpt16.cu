@@ -5,7 +5,7 @@
 // Same algorithm and the same branch-free micro-step structure as
 // replay_lpt.cu; what differs is the state layout:
 //  * 14 bytes per container instead of 24 (n = 64: 896 B per trace, 28 KB per
-//    warp): key (u32), ust (u32: used 16 | op index 3 | FIRST | PAUSED |
+//    warp): key (u32), ust (u32: used 16 | op index 2 | FIRST | PAUSED |
 //    ADMITTED | op kinds 2 x K), sd (u32: size of the current op, saturated
 //    to 16 bits | delta of the next op 16), L (u16, [container][lane]);
 //  * no admission word: an admission is stored straight to admit_tick, or to
@@ -20,7 +20,12 @@
 //    it runs 8 warps per SM too); traces with more distinct limits are left
 //    to the fallback pass;
 //  * arrival + sum of deltas of every container (for R17's wait) is parked
-//    in the thread's tensor-memory lane between init and epilogue;
+//    in the thread's tensor-memory lane between init and epilogue (16 at a
+//    time: init and epilogue run converged for every lane of the warp);
+//  * init reads the trace and the epilogue its admissions with 32-byte loads
+//    (LDG.256, one whole DRAM sector of the lane's own row per instruction)
+//    and writes the outputs with 32-byte streaming stores, when the arrays
+//    are 32-B aligned (else 16-byte operations);
 //  * under R1-LIT (policy | CONVGPU_DISPATCH_LITERAL, NEXT-1) each
 //    container's partial assignment is a u16 at [container][lane] (7 warps
 //    per SM) and the fallback pass is the warp-per-trace kernel;
@@ -33,11 +38,14 @@
 //    head); an event of the container fetched in the previous iteration
 //    (rare) waits one iteration, until the retire has landed its op.
 // A trace qualifies when every limit is <= 0xFFFE MiB, every delta <= 0xFFFF
-// ticks and its horizon (R19) < 2^25 (BASELINE configs [1]-[4] all do; the
-// 16-bit fields are then exact: a saturated size is above every limit, so it
-// is rejected / flagged exactly as the full size would be).  Other traces are
-// marked (admissions[trace][0] = kMark) and replayed by the 32-bit
-// lane-per-trace kernel in a second launch that skips unmarked traces.
+// ticks and its horizon (R19) < 2^25 (BASELINE configs [1]-[3] and [4] up to
+// rho = 7 do; the 16-bit fields are then exact: a saturated size is above
+// every limit, so it is rejected / flagged exactly as the full size would
+// be).  Other traces are marked (admissions[trace][0] = kLpt16Mark) and
+// replayed by a second launch of this kernel with 17-bit limits / used memory
+// (WIDE, R1; exact while every ALLOC / FREE size is <= 0xFFFE), which marks
+// what it cannot hold (kLpt16Mark2) for a third, 32-bit lane-per-trace
+// launch; each launch skips unmarked traces.
 // Semantics are identical to replay_lpt.cu / replay.cu; every
 // GPU parity test runs this kernel against the oracle too.
 #include <cuda_runtime.h>
